@@ -1,0 +1,371 @@
+#!/usr/bin/env python3
+"""Benchmark of the B200 ECL-MST hot path (one JSON line on rank 0).
+
+metric (BASELINE.json): MSF edges/sec and ms/graph; a "step" is one complete
+MSF computation (all hot-path stages: init, threshold, populate, rounds,
+phase 2) over the workload graph, resident in HBM.  Edges/s counts CSR
+entries per second, the paper's throughput convention (Table 2).
+
+Workload at N=1: BASELINE configs[1], the road-network-like graph (C2,
+24M vertices, ~57.6M CSR entries); --config selects another family.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import torch  # noqa: E402
+
+PEAKS_FILE = os.path.join(ROOT, "MEASURED_PEAKS.json")
+PROFILE_SUMMARY = os.path.join(ROOT, "profiles", "ncu_summary_latest.json")
+CONFIG_NAMES = {"grid": "C1", "road": "C2", "rgg": "C3", "rmat": "C4", "uniform": "C5"}
+METRIC = "MSF edges/sec and ms/graph"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=9)     # the paper reports the median of 9 runs
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="road", choices=list(CONFIG_NAMES))
+    ap.add_argument("--size", default="full", choices=["full", "small"])
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-parity", action="store_true")
+    ap.add_argument("--flush-mb", type=int, default=512)
+    return ap.parse_args()
+
+
+# ---------------------------------------------------------------------------
+def dist_env():
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons during the timed region."""
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.gpu = gpu_index
+        self.proc = None
+        self.lines = []
+        self.thread = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--id={self.gpu}", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                 "-lms", "100"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+        except (OSError, ValueError):
+            self.proc = None
+            return
+        self.thread = threading.Thread(target=self._read, daemon=True)
+        self.thread.start()
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.25)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except subprocess.TimeoutExpired:
+            self.proc.kill()
+        if self.thread:
+            self.thread.join(timeout=2)
+        sm, smax, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [p.strip() for p in ln.split(",")]
+            if len(parts) < 9:
+                continue
+            try:
+                sm.append(float(parts[1]))
+                smax.append(float(parts[2]))
+            except ValueError:
+                continue
+            for nm, val in zip(names, parts[5:9]):
+                if val.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None,
+                "sm_max_mhz": max(smax) if smax else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def algorithmic_bytes(n: int, M: int, st: dict) -> dict:
+    """Bytes the method must move per launch.
+
+    init        20 B/vertex  (parent 4 + two key buffers 8+8)
+    populate    8 B/CSR entry (nlist+eweight) + 8 B/vertex (nindex) [+1 B/entry in_mst, phase 1]
+                + per emitted tuple 16 B write + 2x8 B key atomicMin
+                [+ 2x4 B parent gathers per heavy canonical edge, phase 2]
+    pass A      per input tuple 16 B read + 2x4 B parent; per survivor 16 B write + 2x8 B key min
+    pass B      per tuple 16 B read + 2x8 B key reads; per winner 4 B CAS + 1 B mark + 8 B sum
+    """
+    live = st["live"]
+    win = st["winners"]
+    R = len(live)
+    p2 = st["phase2_round"]
+    b = {"init": 20 * n}
+    b["populate"] = (8 * M + 8 * n + M) + 32 * (live[0] if R else 0)
+    passA = passB = 0
+    for g in range(1, R):
+        if g == p2:
+            b["populate"] += 8 * M + 8 * n + 8 * st["heavy_edges"] + 32 * live[g]
+            continue
+        passA += 24 * live[g - 1] + 32 * live[g]
+    for g in range(R):
+        passB += 32 * live[g] + 13 * win[g]
+    b["passA"] = passA
+    b["passB"] = passB
+    b["total"] = sum(b.values())
+    return b
+
+
+def stage_times(st: dict) -> dict:
+    """Split the single kernel's time by the device timestamps (globaltimer)."""
+    t = st["t_ns"]
+    R = st["rounds"]
+    if not t or t[0] == 0 or t[2] == 0:
+        return {}
+    out = {"init_us": (t[1] - t[0]) / 1e3}
+    p2 = st["phase2_round"]
+    prev = t[1]
+    pop = a = bsum = 0.0
+    for g in range(R):
+        ta = t[4 + 2 * g]
+        if g == 0 or g == p2:
+            pop += ta - prev
+        else:
+            a += ta - prev
+        prev = ta
+        tb = t[5 + 2 * g]
+        if tb and g < R - 1:
+            bsum += tb - prev
+            prev = tb
+    out.update(populate_us=pop / 1e3, passA_us=a / 1e3, passB_us=bsum / 1e3, total_us=(t[2] - t[0]) / 1e3)
+    return out
+
+
+def load_peaks():
+    try:
+        with open(PEAKS_FILE) as f:
+            p = json.load(f)
+        return float(p["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except (OSError, KeyError, ValueError):
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def load_traffic():
+    try:
+        with open(PROFILE_SUMMARY) as f:
+            s = json.load(f)
+        return s
+    except (OSError, ValueError):
+        return None
+
+
+# ---------------------------------------------------------------------------
+def run_reference(args, rank, world):
+    """--impl reference: the CPU oracle as it stands, on the host cores."""
+    if rank != 0:
+        return
+    import numpy as np  # noqa: F401
+    import oracle
+    import synth
+    g = synth.make_config(args.config, args.size)
+    n, nindex, nlist, eweight = g.numpy()
+    times = []
+    for i in range(args.warmup + args.steps):
+        t0 = time.perf_counter()
+        oracle.kruskal(n, nindex, nlist, eweight)
+        dt = time.perf_counter() - t0
+        if i >= args.warmup:
+            times.append(dt)
+    ms = 1e3 * sum(times) / len(times)
+    value = g.M / (ms / 1e3)
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": "edges/s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+        "config": {"workload": f"{CONFIG_NAMES[args.config]} {g.name}", "n": g.n, "M": g.M},
+        "cpu_baseline": {"value": value, "unit": "edges/s", "cores": 1, "kind": "oracle",
+                         "sample": f"whole {g.name} graph per step (serial C Kruskal, oracle/kruskal.c)"},
+        "e2e": {"value": value, "unit": "edges/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse()
+    rank, world, local = dist_env()
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+    import paper_conf_sc_fallingsb23_b200 as eclmst
+    import synth
+
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=dev)
+    eclmst.load()   # fails loudly if libeclmst.so is missing
+
+    t_gen = time.perf_counter()
+    g = synth.make_config(args.config, args.size, device=dev)
+    torch.cuda.synchronize()
+    t_gen = time.perf_counter() - t_gen
+    n, M = g.n, g.M
+
+    ws_bytes = eclmst.ecl_mst_workspace_bytes(n, M)
+    ws = torch.empty(ws_bytes, dtype=torch.uint8, device=dev)
+    in_mst = torch.empty(M, dtype=torch.uint8, device=dev)
+    total = torch.empty(1, dtype=torch.int64, device=dev)
+    flush = torch.empty(args.flush_mb << 20, dtype=torch.uint8, device=dev)
+    stream = torch.cuda.current_stream()
+
+    def step():
+        eclmst.ecl_mst_device(n, g.nindex, g.nlist, g.eweight, in_mst_out=in_mst, total_weight_out=total,
+                              workspace=ws, stream=stream)
+
+    for _ in range(max(args.warmup, 3)):
+        flush.zero_()
+        step()
+    torch.cuda.synchronize()
+
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    sampler = ClockSampler(local)
+    sampler.start()
+    if world > 1:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+    wall0 = time.perf_counter()
+    for i in range(args.steps):
+        flush.zero_()                      # L2 flush between timed steps (outside the events)
+        ev[i][0].record(stream)
+        step()
+        ev[i][1].record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        torch.distributed.barrier()
+    wall = time.perf_counter() - wall0
+    clocks = sampler.stop()
+    per_step = [a.elapsed_time(b) for a, b in ev]
+    ms = sum(per_step) / len(per_step)
+    ms_max = ms
+    if world > 1:
+        t = torch.tensor([ms], device=dev)
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        ms_max = float(t.item())
+
+    st = eclmst.ecl_mst_read_stats(ws)
+    result_total = int(total.item())
+
+    # ---- e2e through the host C-ABI call (pinned host buffers, copies timed) ----
+    e2e = None
+    if not args.no_e2e:
+        h_idx = g.nindex.cpu().pin_memory()
+        h_list = g.nlist.cpu().pin_memory()
+        h_w = g.eweight.cpu().pin_memory()
+        h_out = torch.empty(M, dtype=torch.uint8).pin_memory()
+        for _ in range(2):
+            eclmst.ecl_mst(n, h_idx, h_list, h_w, h_out)
+        et = []
+        for _ in range(args.steps):
+            t0 = time.perf_counter()
+            tot_h = eclmst.ecl_mst(n, h_idx, h_list, h_w, h_out)
+            et.append(time.perf_counter() - t0)
+        eclmst.ecl_mst_release_host_cache()
+        e_ms = 1e3 * sum(et) / len(et)
+        if world > 1:
+            t = torch.tensor([e_ms], device=dev)
+            torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+            e_ms = float(t.item())
+        e2e = {"value": world * M / (e_ms / 1e3), "unit": "edges/s",
+               "h2d_bytes_per_step": 8 * (n + 1) + 8 * M, "d2h_bytes_per_step": M + 8,
+               "ms_per_step": e_ms, "same_result": tot_h == result_total}
+
+    if rank != 0:
+        if world > 1:
+            torch.distributed.destroy_process_group()
+        return
+
+    # ---- parity + cpu baseline: the oracle on the same arrays (rank 0, N=1 only) ----
+    parity = None
+    cpu_baseline = None
+    if world == 1 and not (args.no_cpu_baseline and args.no_parity):
+        import numpy as np
+        import oracle
+        hn, hidx, hlist, hw = g.numpy()
+        t0 = time.perf_counter()
+        omask, ototal, _ = oracle.kruskal(hn, hidx, hlist, hw)
+        o_s = time.perf_counter() - t0
+        if not args.no_parity:
+            parity = bool(ototal == result_total and np.array_equal(omask, in_mst.cpu().numpy()))
+        if not args.no_cpu_baseline:
+            cpu_baseline = {"value": M / o_s, "unit": "edges/s", "cores": 1, "kind": "oracle",
+                            "ms": 1e3 * o_s,
+                            "sample": f"whole {g.name} graph, one serial C Kruskal run (oracle/kruskal.c) "
+                                      f"on the GPU box host ({os.cpu_count()} cores present, 1 used)"}
+
+    peak, peak_src = load_peaks()
+    ab = algorithmic_bytes(n, M, st)
+    achieved = ab["total"] / (ms / 1e3) / 1e9
+    prof = load_traffic()
+    traffic = None
+    if prof and prof.get("workload") == g.name:
+        traffic = prof.get("dram_bytes_per_launch")
+    value = world * M / (ms_max / 1e3)
+    line = {
+        "metric": METRIC, "value": value, "unit": "edges/s", "n_gpus": world, "steps": args.steps,
+        "warmup": max(args.warmup, 3), "ms_per_step": ms_max, "higher_is_better": True,
+        "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+        "config": {"workload": f"{CONFIG_NAMES[args.config]} {g.name}", "n": n, "M": M,
+                   "m_undirected": st["canonical_edges"], "parallelism": "replicas" if world > 1 else "single",
+                   "l2": f"inputs ({(8 * M + 8 * n) / 1e6:.0f} MB CSR) exceed L2; plus {args.flush_mb} MB flush "
+                         "between steps"},
+        "ms_per_graph": ms_max, "ms_per_step_all": per_step, "wall_s": wall,
+        "edges_per_s_undirected": world * st["canonical_edges"] / (ms_max / 1e3),
+        "gpu_launches": args.steps,
+        "clocks": clocks,
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                     "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
+                     "kernel": "mst_persistent", "algorithmic_bytes": ab},
+        "cpu_baseline": cpu_baseline,
+        "e2e": e2e,
+        "parity_vs_oracle": parity,
+        "stats": {"rounds": st["rounds"], "filtered": st["filtered"], "threshold": st["threshold"],
+                  "phase2_round": st["phase2_round"], "grid": st["grid"], "msf_edges": st["msf_edges"],
+                  "live": st["live"], "winners": st["winners"], "stage_us": stage_times(st)},
+        "gen_s": t_gen,
+    }
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        torch.distributed.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,136 @@
+/*
+ * ecl_mst.h -- C ABI of the B200-native ECL-MST hot path (libeclmst.so).
+ *
+ * Operation (§3; Alg. 2): the minimum spanning
+ * forest (MSF, P:51, P:63 fn 1) of an undirected graph with 32-bit integer
+ * edge weights given in CSR form with both directions of every edge (P:146,
+ * P:329 fn 2), computed by the edge-centric Kruskal/Boruvka hybrid:
+ * populate a worklist of edges (Alg. 2 L1-11) -> rounds of {find with implicit
+ * path compression, compaction (L17-18), 64-bit
+ * atomicMin of (weight:edge-id) into each representative,
+ * check/join/mark (L27-31)} until the worklist is empty, with a single
+ * weight-threshold filtering step.
+ *
+ * Edge set and ids (readings Q1/Q11): the graph's edges are exactly
+ * the CSR entries j of row u with u < nlist[j] (Alg. 2 L4, "only process in
+ * one direction"); the edge ID of such an edge is j.  Mirror entries and
+ * self-loops are never edges; parallel entries are distinct edges.  Edges are
+ * ordered by (weight as signed int32, id); under that strict order the MSF is
+ * unique, and the library returns exactly it, deterministically.
+ *
+ * Common argument conventions
+ *   n        number of vertices, 0 <= n <= 2^31 - 1.
+ *   M        number of CSR entries = nindex[n], 0 <= M <= 2^32 - 1.
+ *   nindex   int64[n+1], nindex[0] = 0, non-decreasing, nindex[n] = M.
+ *   nlist    int32[M], 0 <= nlist[j] < n: the neighbour of entry j.
+ *   eweight  int32[M]: the weight of entry j (any int32 value).
+ *   in_mst   uint8[M] OUTPUT: 1 iff entry j is the id of an MSF edge, else 0
+ *            (mirror slots are always 0).  Every byte is written.
+ * Ownership: the caller owns every buffer; inputs are only read.  The library
+ * keeps no state between calls except a per-thread last-error string and, for
+ * the host convenience call, a cached device buffer pool (freed by
+ * ecl_mst_release_host_cache).  Calls on distinct workspaces/streams are
+ * independent.
+ */
+#ifndef ECL_MST_H
+#define ECL_MST_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define ECL_MST_ABI_VERSION 1
+
+/* status codes */
+#define ECL_MST_OK 0
+#define ECL_MST_ERR_INVALID (-1)   /* bad argument (null pointer with M > 0, n < 0, ...) */
+#define ECL_MST_ERR_TOO_LARGE (-2) /* n or M beyond the limits above */
+#define ECL_MST_ERR_CUDA (-3)      /* a CUDA call failed; see ecl_mst_last_error() */
+#define ECL_MST_ERR_WORKSPACE (-4) /* workspace too small or misaligned */
+#define ECL_MST_ERR_INPUT (-5)     /* the device found an inconsistent CSR (stats.status) */
+
+#define ECL_MST_MAX_ROUNDS 128     /* global round slots (<= ceil(log2 n)+1 per phase) */
+
+/* knobs; every setting returns the identical MSF (tests check this) */
+typedef struct ecl_mst_options {
+    int32_t filter;          /* -1 auto: filter iff M >= 4n (reading Q6); 0 off; 1 on */
+    int32_t threshold_mode;  /* 0 sampled: 20 weights, c = 4 (reading Q5/Q7); 1 fixed */
+    int32_t threshold;       /* phase 1 takes w < threshold when threshold_mode == 1 */
+    int32_t path_halving;    /* 1 (default) find() halves paths it walks (P:142 reading Q15); 0 off */
+    int32_t max_ctas;        /* 0 = fill the GPU (SMs x resident CTAs); else cap the grid */
+    int32_t reserved;
+    uint64_t seed;           /* seed of the threshold sample */
+} ecl_mst_options;
+
+/* per-run statistics written by the device into the workspace */
+typedef struct ecl_mst_stats {
+    int32_t status;          /* 0 or ECL_MST_ERR_INPUT */
+    int32_t filtered;        /* 1 if two phases ran */
+    int32_t threshold;       /* phase-1 threshold (phase 1: w < threshold) */
+    int32_t rounds;          /* global rounds used (all phases; incl. final empty pass A) */
+    int32_t phase2_round;    /* first global round of phase 2 (-1 if none) */
+    int32_t grid;            /* CTAs of the persistent launch */
+    int32_t block;           /* threads per CTA */
+    int32_t reserved;
+    int64_t total_weight;
+    int64_t msf_edges;
+    int64_t canonical_edges; /* |E| = #{j : u < nlist[j]} */
+    int64_t heavy_edges;     /* canonical edges with w >= threshold (deferred to phase 2) */
+    int64_t live[ECL_MST_MAX_ROUNDS];     /* worklist size after pass A of each global round */
+    int64_t winners[ECL_MST_MAX_ROUNDS];  /* MSF edges added in pass B of each global round */
+    int64_t t_ns[2 * ECL_MST_MAX_ROUNDS + 4]; /* device timestamps (globaltimer) per stage */
+} ecl_mst_stats;
+
+/* Default options (filter auto, sampled threshold, seed 0x5eed, halving on). */
+void ecl_mst_default_options(ecl_mst_options *opts);
+
+/* Bytes of device workspace ecl_mst_device needs for (n, M); 0 if too large.
+ * Layout: header+stats, parent[n] int32,
+ * key[2][n] int64 (double-buffered best-edge slots), worklist int4[M]. */
+size_t ecl_mst_workspace_bytes(int64_t n, int64_t M);
+
+/*
+ * The hot path.  All pointers are DEVICE pointers (current device).  Runs
+ * asynchronously on `stream` (a cudaStream_t; NULL = legacy default stream)
+ * as ONE persistent cooperative kernel: no host round-trips per round.
+ * total_weight_out (device int64*) receives the MSF weight, or INT64_MIN if
+ * the device detected an inconsistent CSR (then stats.status = ERR_INPUT and
+ * in_mst is unspecified).  workspace must be >= ecl_mst_workspace_bytes(n, M)
+ * bytes, 256-byte aligned; its contents on entry are irrelevant.  opts may be
+ * NULL.  Returns ECL_MST_OK or an ECL_MST_ERR_* code for argument / launch
+ * errors (nothing is launched then).
+ */
+int ecl_mst_device(int32_t n, int64_t M, const int64_t *nindex, const int32_t *nlist,
+                   const int32_t *eweight, uint8_t *in_mst_out, int64_t *total_weight_out,
+                   void *workspace, size_t workspace_bytes, const ecl_mst_options *opts,
+                   void *stream);
+
+/* Synchronises `stream`, then copies the statistics of the last run that used
+ * `workspace` to host memory.  Returns ECL_MST_OK or ECL_MST_ERR_CUDA. */
+int ecl_mst_read_stats(const void *workspace, ecl_mst_stats *stats_out, void *stream);
+
+/*
+ * Convenience call with HOST pointers (the paper's "ECL-MST memcpy" variant,
+ * P:325): copies the CSR to the device, runs ecl_mst_device, copies in_mst
+ * back, synchronously.  Pinned host buffers give full PCIe bandwidth.
+ * Returns the MSF weight, or INT64_MIN on any error (ecl_mst_last_error()).
+ */
+int64_t ecl_mst(int32_t n, const int64_t *nindex, const int32_t *nlist,
+                const int32_t *eweight, uint8_t *in_mst_out);
+
+/* Frees the device buffers cached by ecl_mst(). */
+void ecl_mst_release_host_cache(void);
+
+/* Message of the last failed call on this thread ("" if none). */
+const char *ecl_mst_last_error(void);
+
+int ecl_mst_abi_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* ECL_MST_H */

@@ -1,0 +1,185 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the CPU oracle, bit-exact.
+
+The in_mst byte mask and the int64 total weight must equal the oracle's on
+the same seeded inputs (BASELINE.json north_star).
+"""
+import math
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import synth
+from synth import graphs as G
+from tests.fixtures import asymmetric_graph, empty_graph, load_fig2
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def eclmst():
+    import paper_conf_sc_fallingsb23_b200 as m
+    m.load()
+    return m
+
+
+def gpu_run(m, g, **opts):
+    dev = torch.device("cuda:0")
+    gd = g.to(dev)
+    o = m.default_options(**opts) if opts else None
+    mask, total, ws = m.ecl_mst_device(gd.n, gd.nindex, gd.nlist, gd.eweight, options=o)
+    stats = m.ecl_mst_read_stats(ws)
+    return mask.cpu().numpy(), int(total.item()), stats
+
+
+def assert_parity(m, g, **opts):
+    omask, ototal, ocount = oracle.kruskal_graph(g)
+    mask, total, stats = gpu_run(m, g, **opts)
+    assert stats["status"] == 0
+    assert total == ototal, (total, ototal)
+    if not np.array_equal(mask, omask):
+        diff = np.nonzero(mask != omask)[0]
+        raise AssertionError(f"{len(diff)} mask mismatches, first ids {diff[:10]}")
+    assert stats["msf_edges"] == ocount
+    return stats
+
+
+def check_round_bound(g, stats):
+    """<= ceil(log2 n) + 1 rounds per phase incl. the final empty pass A."""
+    bound = math.ceil(math.log2(max(g.n, 2))) + 1
+    r = stats["rounds"]
+    p2 = stats["phase2_round"]
+    if p2 < 0:
+        assert r <= bound + 1, (r, bound)
+    else:
+        assert p2 <= bound + 1 and r - p2 <= bound + 1, (r, p2, bound)
+
+
+def test_fig2(eclmst):
+    g, ids, mst, weight = load_fig2()
+    mask, total, stats = gpu_run(eclmst, g)
+    assert total == weight
+    assert {lab for lab, j in ids.items() if mask[j]} == mst
+    # two iterations that join edges, then the empty final pass
+    assert stats["winners"][:2] == [2, 1]
+
+
+@pytest.mark.parametrize("seed", range(40))
+def test_tiny_adversarial(eclmst, seed):
+    kinds = ["ties", "equal", "two", "full", "uniform"]
+    g = G.random_small(2 + seed % 9, 3 + (seed * 7) % 40, seed=seed, weights=kinds[seed % 5],
+                       multi=seed % 3 == 0, self_loops=seed % 4 == 0)
+    assert_parity(eclmst, g)
+
+
+@pytest.mark.parametrize("weights", ["ties", "two", "full", "uniform", "equal"])
+@pytest.mark.parametrize("n,m", [(1000, 6000), (5000, 2000), (20000, 200000)])
+def test_random_multi_tile(eclmst, weights, n, m):
+    g = G.random_small(n, m, seed=n + m, weights=weights, multi=True, self_loops=True)
+    stats = assert_parity(eclmst, g)
+    check_round_bound(g, stats)
+
+
+@pytest.mark.parametrize("name", list(synth.CONFIGS))
+def test_config_small(eclmst, name):
+    g = synth.make_config(name, "small")
+    stats = assert_parity(eclmst, g)
+    check_round_bound(g, stats)
+
+
+@pytest.mark.parametrize("opts", [
+    dict(filter=0), dict(filter=1), dict(filter=1, threshold_mode=1, threshold=-(1 << 31)),
+    dict(filter=1, threshold_mode=1, threshold=(1 << 31) - 1), dict(filter=1, threshold_mode=1, threshold=0),
+    dict(seed=1), dict(seed=12345), dict(path_halving=0), dict(max_ctas=1), dict(max_ctas=7),
+])
+@pytest.mark.parametrize("name", ["rmat", "uniform", "road"])
+def test_knobs_give_identical_msf(eclmst, name, opts):
+    g = synth.make_config(name, "small")
+    assert_parity(eclmst, g, **opts)
+
+
+def test_two_valued_weights_nontrivial_phase1(eclmst):
+    """Reading Q2: phase 2 must keep canonical ids/directions (tie-heavy)."""
+    for seed in range(6):
+        g = G.random_small(3000, 40000, seed=seed, weights="two")
+        assert_parity(eclmst, g, filter=1, threshold_mode=1, threshold=1)
+
+
+def test_special_graphs(eclmst):
+    assert_parity(eclmst, G.star_graph(1_000_001, seed=1))                # one 1M-degree row
+    assert_parity(eclmst, G.path_graph(200_000))                         # monotone: deep chain
+    assert_parity(eclmst, G.path_graph(200_000, weights=-torch.arange(199_999)))
+    assert_parity(eclmst, G.complete_graph(700, seed=2, weights="ties"))
+    assert_parity(eclmst, G.cycle_graph(99_999, seed=3, weights="ties"))
+    assert_parity(eclmst, asymmetric_graph())
+    # exactly M = 4n: the filter boundary
+    n = 50_000
+    a = torch.arange(n, dtype=torch.int64)
+    u = torch.cat([a, a])
+    v = torch.cat([(a + 1) % n, (a + 2) % n])
+    w = synth.rng.uniform_int31(4, 1, torch.arange(2 * n))
+    g = G.csr_from_undirected(n, u, v, w)
+    assert g.M == 4 * n
+    st = assert_parity(eclmst, g)
+    assert st["filtered"]
+
+
+def test_many_components_and_isolated(eclmst):
+    g = G.random_small(100_000, 30_000, seed=8, weights="ties")  # mostly isolated vertices
+    assert_parity(eclmst, g)
+    g = G.rmat(scale=16, edge_factor=4, seed=8)
+    assert_parity(eclmst, g)
+
+
+def test_degenerate(eclmst):
+    for n in (0, 1, 17):
+        g = empty_graph(n)
+        if n == 0:
+            mask, total, _ = gpu_run(eclmst, g)
+            assert mask.size == 0 and total == 0
+        else:
+            assert_parity(eclmst, g)
+    assert_parity(eclmst, G.path_graph(2, weights=torch.tensor([(1 << 31) - 1])))
+    assert_parity(eclmst, G.random_small(2, 50, seed=1, weights="full", multi=True, self_loops=True))
+
+
+def test_deterministic_and_reusable_workspace(eclmst):
+    g = synth.make_config("rmat", "small").to("cuda:0")
+    a, ta, ws = eclmst.ecl_mst_device(g.n, g.nindex, g.nlist, g.eweight)
+    a = a.clone()
+    ta = int(ta.item())
+    for _ in range(3):
+        b, tb, ws = eclmst.ecl_mst_device(g.n, g.nindex, g.nlist, g.eweight, workspace=ws)
+        assert torch.equal(a, b) and int(tb.item()) == ta
+
+
+def test_host_api_memcpy_variant(eclmst):
+    g = synth.make_config("road", "small")
+    omask, ototal, _ = oracle.kruskal_graph(g)
+    out = torch.empty(g.M, dtype=torch.uint8).pin_memory()
+    total = eclmst.ecl_mst(g.n, g.nindex.pin_memory(), g.nlist.pin_memory(), g.eweight.pin_memory(), out)
+    assert total == ototal
+    assert np.array_equal(out.numpy(), omask)
+    # invalid CSR (neighbour out of range) is reported, not crashed on
+    bad = g.nlist.clone()
+    bad[5] = g.n + 3
+    with pytest.raises(eclmst.EclMstError):
+        eclmst.ecl_mst(g.n, g.nindex, bad, g.eweight, out)
+
+
+def test_device_detects_inconsistent_csr(eclmst):
+    g = synth.make_config("grid", "small").to("cuda:0")
+    bad = g.nindex.clone()
+    bad[-1] += 1   # nindex[n] != M
+    mask, total, ws = eclmst.ecl_mst_device(g.n, bad, g.nlist, g.eweight)
+    st = eclmst.ecl_mst_read_stats(ws)
+    assert st["status"] == -5 and int(total.item()) == -(1 << 63)
+
+
+@pytest.mark.parametrize("name", ["grid", "road"])
+def test_full_size_exact(eclmst, name):
+    """BASELINE configs C1/C2 at full size, whole mask vs the oracle."""
+    g = synth.make_config(name, "full", device="cuda:0").to("cpu")
+    stats = assert_parity(eclmst, g)
+    check_round_bound(g, stats)
