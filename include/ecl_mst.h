@@ -60,6 +60,8 @@ typedef struct ecl_mst_options {
     int32_t threshold_mode;  /* 0 sampled: 20 weights, c = 4 (reading Q5/Q7); 1 fixed */
     int32_t threshold;       /* phase 1 takes w < threshold when threshold_mode == 1 */
     int32_t path_halving;    /* 1 (default) find() halves paths it walks (P:142 reading Q15); 0 off */
+    int32_t atomic_guards;   /* 1 (default) load-compare before each atomicMin; 0 always atomic */
+    int32_t flatten;         /* 1 (default) compress every path once before the phase-2 populate; 0 off */
     int32_t max_ctas;        /* 0 = fill the GPU (SMs x resident CTAs); else cap the grid */
     int32_t reserved;
     uint64_t seed;           /* seed of the threshold sample */
@@ -84,12 +86,13 @@ typedef struct ecl_mst_stats {
     int64_t t_ns[2 * ECL_MST_MAX_ROUNDS + 4]; /* device timestamps (globaltimer) per stage */
 } ecl_mst_stats;
 
-/* Default options (filter auto, sampled threshold, seed 0x5eed, halving on). */
+/* Default options (filter auto, sampled threshold, seed 0x5eed, halving,
+ * guards and flatten on). */
 void ecl_mst_default_options(ecl_mst_options *opts);
 
 /* Bytes of device workspace ecl_mst_device needs for (n, M); 0 if too large.
- * Layout: header+stats, parent[n] int32,
- * key[2][n] int64 (double-buffered best-edge slots), worklist int4[M]. */
+ * Layout: header+stats, key[n] int64 (best-edge
+ * slots), parent[n] int32, two worklists int4[M] (in / out of a pass). */
 size_t ecl_mst_workspace_bytes(int64_t n, int64_t M);
 
 /*

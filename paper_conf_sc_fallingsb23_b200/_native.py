@@ -30,6 +30,8 @@ class EclMstOptions(ctypes.Structure):
         ("threshold_mode", ctypes.c_int32),
         ("threshold", ctypes.c_int32),
         ("path_halving", ctypes.c_int32),
+        ("atomic_guards", ctypes.c_int32),
+        ("flatten", ctypes.c_int32),
         ("max_ctas", ctypes.c_int32),
         ("reserved", ctypes.c_int32),
         ("seed", ctypes.c_uint64),

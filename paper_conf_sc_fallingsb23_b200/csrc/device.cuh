@@ -1,10 +1,10 @@
 // device.cuh -- device building blocks of the ECL-MST hot path (sm_100a).
 //
 // Union-find with implicit path compression (Alg. 2 L15-18),
-// the packed 64-bit (weight:id) best-edge key, lock-free CAS
-// union ("Line 30 ... atomicCAS"), and block-level worklist
-// compaction (warp ballot + one block scan, replacing the paper's per-edge
-// atomicAdd of P:154 "Lines 7 and 18").
+// the packed 64-bit (weight:id) best-edge key, guarded 64-bit
+// atomicMin, and warp-level worklist compaction (ballot + one shared
+// atomicAdd per warp and chunk, replacing the paper's per-edge atomicAdd of
+// P:154 "Lines 7 and 18").
 #pragma once
 
 #include <cstdint>
@@ -14,11 +14,9 @@
 namespace eclmst {
 
 constexpr int kBlock = 512;                  // threads per CTA
-constexpr int kItems = 4;                    // worklist tuples / CSR entries per thread per tile
-constexpr int kTile = kBlock * kItems;       // 2048 per CTA tile
 constexpr int kWarps = kBlock / 32;
-constexpr int kScanSlots = kItems * kWarps;  // per-(item, warp) counts of one tile
-static_assert(kScanSlots == 64, "block_compact scans 64 slots with one warp (2 per lane)");
+constexpr int kItems = 4;                    // tuples / CSR entries per lane per warp chunk
+constexpr int kChunk = 32 * kItems;          // 128 per warp chunk
 constexpr long long kInf = LLONG_MAX;        // "no edge recorded" (reading Q4)
 constexpr unsigned kFull = 0xffffffffu;
 
@@ -35,14 +33,16 @@ __device__ __forceinline__ unsigned long long globaltimer_ns() {
 }
 
 // ---------------------------------------------------------------------------
-// disjoint sets.  parent[] is read through L2 (ld.global.cg): other SMs hook
-// roots with atomicCAS during the check/join pass, and L1 is not coherent.
+// disjoint sets.  parent[] is read through L2 (ld.global.cg): other SMs write
+// it (hooks in pass B, halving anywhere) and L1 is not coherent.  Every
+// parent pointer forms a forest (a vertex is only ever re-pointed to one of
+// its ancestors, or -- a root, once -- to a vertex of another set), so every
+// walk terminates.
 // ---------------------------------------------------------------------------
 
 // Continue a find() from x whose parent px is already loaded.  With halving
 // on, every visited non-root is re-pointed to its grandparent (path halving;
-// benign race: the stored value is always an ancestor, and roots are never
-// written except by the CAS in join()).
+// a benign race: the stored value is always an ancestor).
 __device__ __forceinline__ int find_from(int* __restrict__ parent, int x, int px, bool halving) {
     while (px != x) {
         const int ppx = __ldcg(parent + px);
@@ -58,65 +58,34 @@ __device__ __forceinline__ int find_root(int* __restrict__ parent, int x, bool h
     return find_from(parent, x, __ldcg(parent + x), halving);
 }
 
-// Lock-free union: hook the larger root under the smaller with
-// atomicCAS, retrying from the new parent if another thread hooked it first.
-// The root of every set is therefore its minimum vertex id (reading Q3).
-__device__ __forceinline__ void join(int* __restrict__ parent, int a, int b, bool halving) {
-    while (true) {
-        a = find_root(parent, a, halving);
-        b = find_root(parent, b, halving);
-        if (a == b) return;
-        const int lo = min(a, b), hi = max(a, b);
-        const int old = atomicCAS(parent + hi, hi, lo);
-        if (old == hi) return;
-        a = lo;
-        b = old;
-    }
+// 64-bit atomicMin (L20-21) with the paper's optional guard: a plain
+// L2 load first, skipping the atomic when it cannot lower the slot.
+__device__ __forceinline__ void record_min(long long* slot, long long key, bool guard) {
+    if (!guard || __ldcg(slot) > key) atomicMin(slot, key);
 }
 
-// Guarded 64-bit atomicMin ("atomic guards"): plain L2 load first,
-// skip the atomic if it cannot lower the slot.
-__device__ __forceinline__ void guarded_min(long long* slot, long long key) {
-    if (__ldcg(slot) > key) atomicMin(slot, key);
-}
-
-// ---------------------------------------------------------------------------
-// block-level compaction of one tile: kItems tuples per thread, any order.
-// Returns the number kept (block-uniform) and writes them to out[0, kept).
-// s_cnt must hold kScanSlots + 1 ints.
-// ---------------------------------------------------------------------------
-__device__ __forceinline__ int block_compact(const int4 (&t)[kItems], const bool (&keep)[kItems],
-                                             int4* __restrict__ out, int* s_cnt) {
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    unsigned mask[kItems];
+// Warp-level compaction of one chunk (kItems tuples per lane, any order):
+// one shared-memory atomicAdd per warp reserves the output range.
+__device__ __forceinline__ int warp_emit(const int4 (&t)[kItems], const bool (&keep)[kItems],
+                                         int4* __restrict__ out, int* s_out) {
+    const int lane = threadIdx.x & 31;
+    unsigned m[kItems];
+    int off[kItems];
+    int tot = 0;
 #pragma unroll
     for (int i = 0; i < kItems; ++i) {
-        mask[i] = __ballot_sync(kFull, keep[i]);
-        if (lane == 0) s_cnt[i * kWarps + warp] = __popc(mask[i]);
+        m[i] = __ballot_sync(kFull, keep[i]);
+        off[i] = tot;
+        tot += __popc(m[i]);
     }
-    __syncthreads();
-    if (warp == 0) {
-        const int a = s_cnt[2 * lane], b = s_cnt[2 * lane + 1];
-        const int s = a + b;
-        int incl = s;
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const int y = __shfl_up_sync(kFull, incl, o);
-            if (lane >= o) incl += y;
-        }
-        const int excl = incl - s;
-        s_cnt[2 * lane] = excl;
-        s_cnt[2 * lane + 1] = excl + a;
-        if (lane == 31) s_cnt[kScanSlots] = incl;
-    }
-    __syncthreads();
+    int base = 0;
+    if (lane == 0 && tot) base = atomicAdd(s_out, tot);
+    base = __shfl_sync(kFull, base, 0);
     const unsigned lt = (1u << lane) - 1u;
 #pragma unroll
     for (int i = 0; i < kItems; ++i)
-        if (keep[i]) __stcg(out + s_cnt[i * kWarps + warp] + __popc(mask[i] & lt), t[i]);
-    const int kept = s_cnt[kScanSlots];
-    __syncthreads();
-    return kept;
+        if (keep[i]) __stcg(out + base + off[i] + __popc(m[i] & lt), t[i]);
+    return tot;
 }
 
 // warp-cooperative 32-ary search: largest r in [0, n) with nindex[r] <= x.

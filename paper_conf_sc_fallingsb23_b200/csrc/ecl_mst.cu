@@ -3,34 +3,41 @@
 //
 // One persistent cooperative kernel per MSF (no host round-trips per round,
 // replacing the paper's host while-loop with a cudaMemcpy per iteration,
-// P:86-88).  Grid = SMs x resident CTAs; CTA b owns CSR entries
-// [b*chunk, (b+1)*chunk) and the same slice of the worklist, which it
-// compacts in place round after round.  Stages, separated by grid barriers:
+// P:86-88).  Grid = SMs x resident CTAs; every warp owns a contiguous
+// range of CSR entries, every CTA the union of its warps' ranges and the same
+// slice of the two worklists.  Warps work independently (warp-level
+// compaction, no CTA barriers inside a pass); stages are separated by grid
+// barriers:
 //
-//   init      Alg. 1: parent[v] = v, both best-edge buffers = inf;
-//             block 0 draws the filter threshold.
-//   populate  Alg. 2 L1-11 over the CTA's CSR range (edge-balanced), FUSED
+//   init      Alg. 1: parent[v] = v, key[v] = inf; block 0 draws the
+//             filter threshold; each warp finds the row of its
+//             first CSR entry.
+//   populate  Alg. 2 L1-11 over the warp's CSR range (edge-balanced), FUSED
 //             with round 0 of L14-21 (all endpoints are roots then, so the
 //             find is the identity and nothing is dropped): emit <u,v,w,id>
 //             for u < v (L4) meeting the threshold (L6), atomicMin the key
 //             into both endpoints.  Phase 2 re-reads the CSR for the
 //             heavy edges, replaces endpoints by set(u), set(v), drops
 //             intra-set edges (the filter) and records keys the same way.
-//   pass B    L27-31: edge whose key won at either endpoint -> join (CAS),
-//             mark in_mst[id], add its weight.
+//   pass B    L27-31: an edge whose key won at endpoint p hooks p under the
+//             other endpoint (Boruvka hooking: each representative is written
+//             by exactly one edge, so no CAS is needed; a mutual pair keeps
+//             its smaller end as root), marks in_mst[id] and adds its weight.
+//             The winning edge of p also resets key[p] (L34-37 fused: an edge
+//             that lost at p compares unequal to both the old minimum and to
+//             inf, so the early reset cannot change any decision).
 //   pass A    L14-23 of the next round: find (implicit path compression,
-//             L15-18), drop p == q, keep <p,q,w,id>, guarded atomicMin into
-//             the OTHER key buffer; also resets the previous buffer at the
-//             tuple's stored endpoints, which are exactly the slots written
-//             last round (L34-37 fused away).
+//             L15-18), drop p == q, keep <p,q,w,id> in the other worklist,
+//             atomicMin the key into both representatives.
+//   flatten   before phase 2: parent[v] = find(v) for every v.
 //
-// Loop: populate ; while (live > 0) { B ; A } per phase.
+// Loop per phase: populate ; while (live > 0) { B ; A }.
 #include <cooperative_groups.h>
 #include <cuda_runtime.h>
 
 #include <climits>
-#include <cstdint>
 #include <cstdarg>
+#include <cstdint>
 #include <cstdio>
 #include <cstring>
 #include <mutex>
@@ -51,7 +58,7 @@ struct Internal {
 };
 
 struct Layout {
-    size_t stats, internal, parent, key0, key1, wl, total;
+    size_t stats, internal, key, parent, wl0, wl1, total;
 };
 
 static inline size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
@@ -61,10 +68,10 @@ static inline Layout layout_for(int64_t n, int64_t M) {
     size_t off = 0;
     L.stats = off;    off = align_up(off + sizeof(ecl_mst_stats), 256);
     L.internal = off; off = align_up(off + sizeof(Internal), 256);
-    L.key0 = off;     off = align_up(off + sizeof(long long) * (size_t)n, 256);
-    L.key1 = off;     off = align_up(off + sizeof(long long) * (size_t)n, 256);
+    L.key = off;      off = align_up(off + sizeof(long long) * (size_t)n, 256);
     L.parent = off;   off = align_up(off + sizeof(int) * (size_t)n, 256);
-    L.wl = off;       off = align_up(off + sizeof(int4) * (size_t)M, 256);
+    L.wl0 = off;      off = align_up(off + sizeof(int4) * (size_t)M, 256);
+    L.wl1 = off;      off = align_up(off + sizeof(int4) * (size_t)M, 256);
     L.total = off;
     return L;
 }
@@ -72,7 +79,7 @@ static inline Layout layout_for(int64_t n, int64_t M) {
 struct Params {
     int n;
     long long M;
-    long long chunk;                  // CSR entries per CTA (multiple of kItems)
+    long long sub;                    // CSR entries per warp (multiple of kItems)
     const long long* __restrict__ nindex;
     const int* __restrict__ nlist;
     const int* __restrict__ eweight;
@@ -80,21 +87,23 @@ struct Params {
     long long* total_out;
     ecl_mst_stats* st;
     Internal* in;
+    long long* key;
     int* parent;
-    long long* key0;
-    long long* key1;
-    int4* wl;
+    int4* wl0;
+    int4* wl1;
     unsigned long long seed;
     int filter_mode;
     int threshold_mode;
     int threshold_value;
     int halving;
+    int guards;
+    int flatten;
     int vec_ok;
 };
 
-// inclusive max-scan of a blocked tile (kItems consecutive values per thread)
-__device__ __forceinline__ void block_max_scan(int (&m)[kItems], int* s_warp) {
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+// inclusive max-scan over a warp's chunk (kItems consecutive values per lane)
+__device__ __forceinline__ void warp_max_scan(int (&m)[kItems]) {
+    const int lane = threadIdx.x & 31;
 #pragma unroll
     for (int k = 1; k < kItems; ++k) m[k] = max(m[k], m[k - 1]);
     int incl = m[kItems - 1];
@@ -105,88 +114,89 @@ __device__ __forceinline__ void block_max_scan(int (&m)[kItems], int* s_warp) {
     }
     int excl = __shfl_up_sync(kFull, incl, 1);
     if (lane == 0) excl = INT_MIN;
-    if (lane == 31) s_warp[warp] = incl;
-    __syncthreads();
-    int pre = excl;
-    for (int w = 0; w < warp; ++w) pre = max(pre, s_warp[w]);
 #pragma unroll
-    for (int k = 0; k < kItems; ++k) m[k] = max(m[k], pre);
-    __syncthreads();
+    for (int k = 0; k < kItems; ++k) m[k] = max(m[k], excl);
 }
 
-// Alg. 2 L1-11 (+ round 0 of L14-21).  PH = 1: light edges; PH = 2: heavy
-// edges with set() endpoints and the cycle filter.
+// Alg. 2 L1-11 (+ round 0 of L14-21) over one warp's CSR range [wb, we).
+// PH = 1: light edges; PH = 2: heavy edges with set() endpoints and the
+// cycle filter.
 template <int PH>
-__device__ __forceinline__ int populate(const Params& P, long long j_begin, long long j_end, int r_first,
-                                        long long* __restrict__ Kc, bool filtered, int T, int* s_mark,
-                                        int* s_cnt, long long& canon_cnt, long long& heavy_cnt, int& err) {
-    const int tid = threadIdx.x;
-    const bool halving = P.halving != 0;
-    int4* seg = P.wl + j_begin;
-    int cnt = 0;
+__device__ __forceinline__ void populate(const Params& P, long long wb, long long we, int r_first,
+                                         bool filtered, int T, int* s_mark, int4* __restrict__ out, int* s_out,
+                                         long long& canon_cnt, long long& heavy_cnt, int& err) {
+    const int lane = threadIdx.x & 31;
+    const bool halving = P.halving != 0, guard = P.guards != 0;
+    long long* __restrict__ K = P.key;
     int r_cur = r_first;
-    for (long long t0 = j_begin; t0 < j_end; t0 += kTile) {
-        const long long t1 = min(t0 + (long long)kTile, j_end);
-        const int len = (int)(t1 - t0);
-        const bool need_carry = t1 < j_end;
-
-        // --- row of every entry: mark row starts inside the tile, then max-scan
-        for (int i = tid; i < kTile; i += kBlock) s_mark[i] = (i == 0) ? r_cur : -1;
-        __syncthreads();
-        int carry = r_cur;
-        for (long long rb = (long long)r_cur + 1;; rb += kBlock) {
-            const long long r = rb + tid;
-            bool active = false;
-            if (r < P.n) {
-                const long long s = __ldg(P.nindex + r);
-                if (s < t1) {
-                    active = true;
-                    if (s >= t0) atomicMax(&s_mark[s - t0], (int)r);
-                    else err = 1;   // nindex decreasing
-                } else if (s == t1 && need_carry) {
-                    active = true;
-                }
-            }
-            const int na = __syncthreads_count(active);
-            if (na > 0) carry = (int)(rb + na - 1);
-            if (na < kBlock) break;
-        }
-
-        const int p0 = tid * kItems;
-        int vv[kItems], ww[kItems];
+    for (long long c0 = wb; c0 < we; c0 += kChunk) {
+        const long long c1 = min(c0 + (long long)kChunk, we);
+        const int len = (int)(c1 - c0);
+        const bool need_carry = c1 < we;
+        const int p0 = lane * kItems;
         const bool full = p0 + kItems <= len;
+
+        // stream the chunk's entries first (independent of the row search)
+        int vv[kItems], ww[kItems];
         if (P.vec_ok && full) {
-            const int4 a = __ldcs(reinterpret_cast<const int4*>(P.nlist + t0 + p0));
-            const int4 b = __ldcs(reinterpret_cast<const int4*>(P.eweight + t0 + p0));
+            const int4 a = __ldcs(reinterpret_cast<const int4*>(P.nlist + c0 + p0));
+            const int4 b = __ldcs(reinterpret_cast<const int4*>(P.eweight + c0 + p0));
             vv[0] = a.x; vv[1] = a.y; vv[2] = a.z; vv[3] = a.w;
             ww[0] = b.x; ww[1] = b.y; ww[2] = b.z; ww[3] = b.w;
         } else {
 #pragma unroll
             for (int k = 0; k < kItems; ++k) {
                 const bool ok = p0 + k < len;
-                vv[k] = ok ? __ldcs(P.nlist + t0 + p0 + k) : -1;
-                ww[k] = ok ? __ldcs(P.eweight + t0 + p0 + k) : 0;
+                vv[k] = ok ? __ldcs(P.nlist + c0 + p0 + k) : -1;
+                ww[k] = ok ? __ldcs(P.eweight + c0 + p0 + k) : 0;
             }
         }
-        if (PH == 1) {   // every in_mst byte is written once, here (Alg. 1 "not in MST")
-            if (P.vec_ok && full) {
-                __stcs(reinterpret_cast<unsigned*>(P.in_mst + t0 + p0), 0u);
-            } else {
+
+        // row of every entry: mark row starts inside the chunk, then max-scan
 #pragma unroll
-                for (int k = 0; k < kItems; ++k)
-                    if (p0 + k < len) P.in_mst[t0 + p0 + k] = 0;
+        for (int i = lane; i < kChunk; i += 32) s_mark[i] = (i == 0) ? r_cur : -1;
+        __syncwarp();
+        int carry = r_cur;
+        for (long long rb = (long long)r_cur + 1;; rb += 32) {
+            const long long r = rb + lane;
+            bool active = false;
+            if (r < P.n) {
+                const long long s = __ldg(P.nindex + r);
+                if (s < c1) {
+                    active = true;
+                    if (s >= c0) atomicMax(&s_mark[s - c0], (int)r);
+                    else err = 1;   // nindex decreasing
+                } else if (s == c1 && need_carry) {
+                    active = true;
+                }
             }
+            const int na = __popc(__ballot_sync(kFull, active));
+            if (na > 0) carry = (int)(rb + na - 1);
+            if (na < 32) break;
         }
+        __syncwarp();
         int row[kItems];
 #pragma unroll
         for (int k = 0; k < kItems; ++k) row[k] = s_mark[p0 + k];
-        block_max_scan(row, s_cnt);
+        __syncwarp();
+        warp_max_scan(row);
+
+        if (PH == 1) {   // every in_mst byte is written once, here (Alg. 1 "not in MST")
+            if (P.vec_ok && full) {
+                __stcs(reinterpret_cast<unsigned*>(P.in_mst + c0 + p0), 0u);
+            } else {
+#pragma unroll
+                for (int k = 0; k < kItems; ++k)
+                    if (p0 + k < len) P.in_mst[c0 + p0 + k] = 0;
+            }
+        }
 
         int4 t[kItems];
         bool keep[kItems];
+        int prev_u = -1, prev_p = -1;
 #pragma unroll
         for (int k = 0; k < kItems; ++k) {
-            const long long j = t0 + p0 + k;
+            const long long j = c0 + p0 + k;
             const bool valid = p0 + k < len;
             const int u = row[k], v = vv[k], w = ww[k];
             const bool in_range = (unsigned)v < (unsigned)P.n;
@@ -200,38 +210,54 @@ __device__ __forceinline__ int populate(const Params& P, long long j_begin, long
                 heavy_cnt += (canon && heavy);
                 kk = canon && !heavy;
             } else if (canon && filtered && w >= T) {
-                p = find_root(P.parent, u, halving);              // set(v), set(n)
-                q = find_root(P.parent, v, halving);
+                p = (u == prev_u) ? prev_p : find_root(P.parent, u, halving);   // set(v)
+                prev_u = u;
+                prev_p = p;
+                q = find_root(P.parent, v, halving);                            // set(n)
                 kk = p != q;                                      // filtered out otherwise
-            }
-            if (kk) {
-                const long long key = make_key(w, (unsigned)j);   // L19 val <- e_w : e_id
-                guarded_min(Kc + p, key);                         // L20
-                guarded_min(Kc + q, key);                         // L21
             }
             t[k] = make_int4(p, q, w, (int)(unsigned)j);
             keep[k] = kk;
         }
-        cnt += block_compact(t, keep, seg + cnt, s_cnt);         // L7 / L18
+        // L20: the lane's entries come in row order, so merge equal p first
+        long long best = kInf;
+        int bp = -1;
+#pragma unroll
+        for (int k = 0; k < kItems; ++k) {
+            if (!keep[k]) continue;
+            const long long key = make_key(t[k].z, (unsigned)t[k].w);   // L19 val <- e_w : e_id
+            if (t[k].x != bp) {
+                if (bp >= 0) record_min(K + bp, best, guard);
+                bp = t[k].x;
+                best = key;
+            } else {
+                best = min(best, key);
+            }
+        }
+        if (bp >= 0) record_min(K + bp, best, guard);
+#pragma unroll
+        for (int k = 0; k < kItems; ++k)                          // L21
+            if (keep[k]) record_min(K + t[k].y, make_key(t[k].z, (unsigned)t[k].w), guard);
+        warp_emit(t, keep, out, s_out);                          // L7
         r_cur = carry;
     }
-    return cnt;
 }
 
-// L14-23 of round g (> 0 within a phase), with L34-37 of round g-1 fused in.
-__device__ __forceinline__ int passA(const Params& P, int4* __restrict__ seg, int cnt,
-                                     long long* __restrict__ Kc, long long* __restrict__ Kp, int* s_cnt) {
-    const bool halving = P.halving != 0;
+// L14-23 of one round over the CTA's worklist slice: in[0, cnt) -> out.
+__device__ __forceinline__ void passA(const Params& P, const int4* __restrict__ in, int cnt,
+                                      int4* __restrict__ out, int* s_out) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const bool halving = P.halving != 0, guard = P.guards != 0;
     int* __restrict__ parent = P.parent;
-    int wp = 0;
-    for (int base = 0; base < cnt; base += kTile) {
+    long long* __restrict__ K = P.key;
+    for (int c = warp * kChunk; c < cnt; c += kWarps * kChunk) {
         int4 t[kItems];
         bool keep[kItems];
 #pragma unroll
         for (int i = 0; i < kItems; ++i) {
-            const int idx = base + i * kBlock + (int)threadIdx.x;
+            const int idx = c + i * 32 + lane;
             keep[i] = idx < cnt;
-            t[i] = keep[i] ? __ldcg(seg + idx) : make_int4(0, 0, 0, 0);
+            t[i] = keep[i] ? __ldcs(in + idx) : make_int4(0, 0, 0, 0);
         }
         int px[kItems], qx[kItems];
 #pragma unroll
@@ -242,63 +268,66 @@ __device__ __forceinline__ int passA(const Params& P, int4* __restrict__ seg, in
             }
         }
 #pragma unroll
-        for (int i = 0; i < kItems; ++i) {   // reset last round's slots (L35-36)
-            if (keep[i]) {
-                if (__ldcg(Kp + t[i].x) != kInf) __stcg(Kp + t[i].x, kInf);
-                if (__ldcg(Kp + t[i].y) != kInf) __stcg(Kp + t[i].y, kInf);
-            }
-        }
-#pragma unroll
         for (int i = 0; i < kItems; ++i) {
             if (keep[i]) {
                 const int p = find_from(parent, t[i].x, px[i], halving);   // L15
                 const int q = find_from(parent, t[i].y, qx[i], halving);   // L16
                 keep[i] = p != q;                                          // L17
-                if (keep[i]) {
-                    const long long key = make_key(t[i].z, (unsigned)t[i].w);
-                    guarded_min(Kc + p, key);
-                    guarded_min(Kc + q, key);
-                    t[i].x = p;    // L18: implicit path compression
-                    t[i].y = q;
-                }
+                t[i].x = p;                                                // L18: implicit
+                t[i].y = q;                                                //      path compression
             }
         }
-        wp += block_compact(t, keep, seg + wp, s_cnt);
+#pragma unroll
+        for (int i = 0; i < kItems; ++i) {
+            if (keep[i]) {
+                const long long key = make_key(t[i].z, (unsigned)t[i].w); // L19
+                record_min(K + t[i].x, key, guard);                       // L20
+                record_min(K + t[i].y, key, guard);                       // L21
+            }
+        }
+        warp_emit(t, keep, out, s_out);                                   // L18
     }
-    return wp;
 }
 
-// L27-31: check, join, mark.
-__device__ __forceinline__ void passB(const Params& P, const int4* __restrict__ seg, int cnt,
-                                      const long long* __restrict__ Kc, long long& wsum, long long& wcnt) {
-    const bool halving = P.halving != 0;
-    for (int base = 0; base < cnt; base += kTile) {
+// L27-31 (+ L34-37): check, join, mark over the CTA's worklist slice.
+__device__ __forceinline__ void passB(const Params& P, const int4* __restrict__ wl, int cnt,
+                                      long long& wsum, long long& wcnt) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    int* __restrict__ parent = P.parent;
+    long long* __restrict__ K = P.key;
+    for (int c = warp * kChunk; c < cnt; c += kWarps * kChunk) {
         int4 t[kItems];
         bool ok[kItems];
 #pragma unroll
         for (int i = 0; i < kItems; ++i) {
-            const int idx = base + i * kBlock + (int)threadIdx.x;
+            const int idx = c + i * 32 + lane;
             ok[i] = idx < cnt;
-            t[i] = ok[i] ? __ldcg(seg + idx) : make_int4(0, 0, 0, 0);
+            t[i] = ok[i] ? __ldcg(wl + idx) : make_int4(0, 0, 0, 0);
         }
         long long kp[kItems], kq[kItems];
 #pragma unroll
         for (int i = 0; i < kItems; ++i) {
             if (ok[i]) {
-                kp[i] = __ldcg(Kc + t[i].x);
-                kq[i] = __ldcg(Kc + t[i].y);
+                kp[i] = __ldcg(K + t[i].x);
+                kq[i] = __ldcg(K + t[i].y);
             }
         }
 #pragma unroll
         for (int i = 0; i < kItems; ++i) {
-            if (ok[i]) {
-                const long long key = make_key(t[i].z, (unsigned)t[i].w);
-                if (kp[i] == key || kq[i] == key) {               // L29
-                    join(P.parent, t[i].x, t[i].y, halving);      // L30
-                    P.in_mst[(unsigned)t[i].w] = 1;               // L31
-                    wsum += t[i].z;
-                    wcnt += 1;
-                }
+            if (!ok[i]) continue;
+            const long long key = make_key(t[i].z, (unsigned)t[i].w);
+            const bool wp = kp[i] == key, wq = kq[i] == key;          // L29
+            if (wp || wq) {
+                const int p = t[i].x, q = t[i].y;
+                // L30 join: each set hooks along its own lightest edge;
+                // a mutual pair keeps the smaller representative as root.
+                if (wp && !(wq && p < q)) __stcg(parent + p, q);
+                if (wq && !(wp && q < p)) __stcg(parent + q, p);
+                if (wp) __stcg(K + p, kInf);                           // L35
+                if (wq) __stcg(K + q, kInf);                           // L36
+                P.in_mst[(unsigned)t[i].w] = 1;                        // L31
+                wsum += t[i].z;
+                wcnt += 1;
             }
         }
     }
@@ -311,34 +340,30 @@ __device__ __forceinline__ void stamp(const Params& P, int slot) {
 
 __global__ void __launch_bounds__(kBlock, 2) mst_persistent(Params P) {
     cg::grid_group grid = cg::this_grid();
-    __shared__ int s_mark[kTile];
-    __shared__ int s_cnt[kScanSlots + 1];
-    __shared__ int s_row;
+    __shared__ int s_mark[kWarps][kChunk];
+    __shared__ int s_out;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const bool b0 = blockIdx.x == 0;
     ecl_mst_stats* st = P.st;
     const long long t_start = (b0 && tid == 0) ? (long long)globaltimer_ns() : 0;
-    const long long j_begin = min(P.M, (long long)blockIdx.x * P.chunk);
-    const long long j_end = min(P.M, j_begin + P.chunk);
+    const long long cta_begin = min(P.M, (long long)blockIdx.x * kWarps * P.sub);
+    const long long wb = min(P.M, cta_begin + warp * P.sub);
+    const long long we = min(P.M, wb + P.sub);
     int err = 0;
 
     // ---------------- init (Alg. 1) ----------------
     for (long long v = (long long)blockIdx.x * kBlock + tid; v < P.n; v += (long long)gridDim.x * kBlock) {
         P.parent[v] = (int)v;
-        P.key0[v] = kInf;
-        P.key1[v] = kInf;
+        P.key[v] = kInf;
     }
-    if (warp == 0) {
-        const int r = (j_begin < j_end) ? warp_row_of(P.nindex, P.n, j_begin) : 0;
-        if (lane == 0) s_row = r;
-    }
+    const int r_first = (wb < we) ? warp_row_of(P.nindex, P.n, wb) : 0;
     if (b0) {
         long long* words = reinterpret_cast<long long*>(st);
         for (int i = tid; i < (int)(sizeof(ecl_mst_stats) / 8); i += kBlock) words[i] = 0;
         __syncthreads();
         if (warp == 1) {
             // filter decision (readings Q5-Q7)
-            bool filtered = P.filter_mode < 0 ? (P.M >= 4LL * P.n) : (P.filter_mode != 0);
+            const bool filtered = P.filter_mode < 0 ? (P.M >= 4LL * P.n) : (P.filter_mode != 0);
             int T = INT_MAX;
             if (filtered) {
                 if (P.threshold_mode == 1) {
@@ -372,7 +397,6 @@ __global__ void __launch_bounds__(kBlock, 2) mst_persistent(Params P) {
         if (tid == 0) P.in->done = 0u;
     }
     grid.sync();
-    const int r_first = s_row;
     const bool filtered = __ldcg(&st->filtered) != 0;
     const int T = __ldcg(&st->threshold);
     if (b0 && tid == 0) {
@@ -381,21 +405,31 @@ __global__ void __launch_bounds__(kBlock, 2) mst_persistent(Params P) {
     }
 
     long long canon_cnt = 0, heavy_cnt = 0, wsum = 0, wcnt = 0;
-    int4* seg = P.wl + j_begin;
-    int g = 0, cnt = 0;
+    int4* wl[2] = {P.wl0 + cta_begin, P.wl1 + cta_begin};
+    int cur = 0, g = 0, cnt = 0;
     bool overflow = false;
     for (int ph = 1; ph <= 2 && !overflow; ++ph) {
         if (ph == 2) {
             if (!filtered || __ldcg(&st->heavy_edges) == 0) break;
             if (g + 1 >= ECL_MST_MAX_ROUNDS) { overflow = true; break; }
+            if (P.flatten) {   // compress every path once: phase-2 finds become one hop
+                for (long long v = (long long)blockIdx.x * kBlock + tid; v < P.n; v += (long long)gridDim.x * kBlock) {
+                    const int r = find_root(P.parent, (int)v, true);
+                    if (r != (int)v) __stcg(P.parent + v, r);
+                }
+                grid.sync();
+            }
             ++g;
             if (b0 && tid == 0) st->phase2_round = g;
         }
-        long long* Kc = (g & 1) ? P.key1 : P.key0;
+        if (tid == 0) s_out = 0;
+        __syncthreads();
         if (ph == 1)
-            cnt = populate<1>(P, j_begin, j_end, r_first, Kc, filtered, T, s_mark, s_cnt, canon_cnt, heavy_cnt, err);
+            populate<1>(P, wb, we, r_first, filtered, T, s_mark[warp], wl[cur], &s_out, canon_cnt, heavy_cnt, err);
         else
-            cnt = populate<2>(P, j_begin, j_end, r_first, Kc, filtered, T, s_mark, s_cnt, canon_cnt, heavy_cnt, err);
+            populate<2>(P, wb, we, r_first, filtered, T, s_mark[warp], wl[cur], &s_out, canon_cnt, heavy_cnt, err);
+        __syncthreads();
+        cnt = s_out;
         if (tid == 0 && cnt) atomicAdd(reinterpret_cast<unsigned long long*>(&st->live[g]), (unsigned long long)cnt);
         if (ph == 1) {
             const long long c = warp_sum(canon_cnt), h = warp_sum(heavy_cnt);
@@ -407,16 +441,18 @@ __global__ void __launch_bounds__(kBlock, 2) mst_persistent(Params P) {
         long long L = __ldcg(&st->live[g]);
         while (L > 0) {
             const long long w0 = wcnt;
-            passB(P, seg, cnt, Kc, wsum, wcnt);
+            passB(P, wl[cur], cnt, wsum, wcnt);
             const long long d = warp_sum(wcnt - w0);
             if (lane == 0 && d) atomicAdd(reinterpret_cast<unsigned long long*>(&st->winners[g]), (unsigned long long)d);
+            if (tid == 0) s_out = 0;
             grid.sync();
             stamp(P, 5 + 2 * g);
             if (g + 1 >= ECL_MST_MAX_ROUNDS) { overflow = true; break; }
             ++g;
-            long long* Kp = Kc;
-            Kc = (g & 1) ? P.key1 : P.key0;
-            cnt = passA(P, seg, cnt, Kc, Kp, s_cnt);
+            passA(P, wl[cur], cnt, wl[cur ^ 1], &s_out);
+            cur ^= 1;
+            __syncthreads();
+            cnt = s_out;
             if (tid == 0 && cnt) atomicAdd(reinterpret_cast<unsigned long long*>(&st->live[g]), (unsigned long long)cnt);
             grid.sync();
             stamp(P, 4 + 2 * g);
@@ -511,6 +547,8 @@ void ecl_mst_default_options(ecl_mst_options* o) {
     o->threshold_mode = 0;
     o->threshold = 0;
     o->path_halving = 1;
+    o->atomic_guards = 1;
+    o->flatten = 1;
     o->max_ctas = 0;
     o->seed = 0x5eedull;
 }
@@ -548,23 +586,27 @@ int ecl_mst_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t* n
     DevInfo di;
     int rc = device_info(&di);
     if (rc) return rc;
-    long long G = (long long)di.sms * di.occ;
-    const long long tiles = (M + kTile - 1) / kTile;
-    if (G > tiles) G = tiles;
+    const long long max_g = (long long)di.sms * di.occ;
+    long long G = max_g;
+    const long long chunks = (M + kChunk - 1) / kChunk;
+    if (G * kWarps > chunks) G = (chunks + kWarps - 1) / kWarps;   // small graphs: fewer CTAs
     if (o.max_ctas > 0 && G > o.max_ctas) G = o.max_ctas;
     if (G > kMaxGrid) G = kMaxGrid;
     if (G < 1) G = 1;
-    // per-CTA counts are int: keep a CTA's slice below 2^30 entries
-    const long long min_g = (M + (1LL << 30) - 1) >> 30;
-    if (G < min_g) G = min_g;
-    if (G > (long long)di.sms * di.occ) return fail(ECL_MST_ERR_TOO_LARGE, "graph needs more CTAs than fit");
-    long long chunk = (M + G - 1) / G;
-    chunk = (chunk + kItems - 1) / kItems * kItems;
+    long long sub = (M + G * kWarps - 1) / (G * kWarps);
+    sub = (sub + kItems - 1) / kItems * kItems;
+    // per-CTA worklist counts are int: keep a CTA's slice below 2^30 entries
+    while (sub * kWarps >= (1LL << 30)) {
+        if (G >= max_g) return fail(ECL_MST_ERR_TOO_LARGE, "graph needs more CTAs than fit");
+        ++G;
+        sub = (M + G * kWarps - 1) / (G * kWarps);
+        sub = (sub + kItems - 1) / kItems * kItems;
+    }
 
     Params P;
     P.n = n;
     P.M = M;
-    P.chunk = chunk;
+    P.sub = sub;
     P.nindex = reinterpret_cast<const long long*>(nindex);
     P.nlist = nlist;
     P.eweight = eweight;
@@ -572,15 +614,17 @@ int ecl_mst_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t* n
     P.total_out = reinterpret_cast<long long*>(total_weight_out);
     P.st = reinterpret_cast<ecl_mst_stats*>(ws + L.stats);
     P.in = reinterpret_cast<Internal*>(ws + L.internal);
+    P.key = reinterpret_cast<long long*>(ws + L.key);
     P.parent = reinterpret_cast<int*>(ws + L.parent);
-    P.key0 = reinterpret_cast<long long*>(ws + L.key0);
-    P.key1 = reinterpret_cast<long long*>(ws + L.key1);
-    P.wl = reinterpret_cast<int4*>(ws + L.wl);
+    P.wl0 = reinterpret_cast<int4*>(ws + L.wl0);
+    P.wl1 = reinterpret_cast<int4*>(ws + L.wl1);
     P.seed = o.seed;
     P.filter_mode = o.filter < 0 ? -1 : (o.filter ? 1 : 0);
     P.threshold_mode = o.threshold_mode;
     P.threshold_value = o.threshold;
     P.halving = o.path_halving ? 1 : 0;
+    P.guards = o.atomic_guards ? 1 : 0;
+    P.flatten = o.flatten ? 1 : 0;
     P.vec_ok = (reinterpret_cast<uintptr_t>(nlist) % 16 == 0) && (reinterpret_cast<uintptr_t>(eweight) % 16 == 0) &&
                (reinterpret_cast<uintptr_t>(in_mst_out) % 4 == 0);
     void* args[] = {&P};

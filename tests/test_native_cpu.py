@@ -34,7 +34,7 @@ def test_exports_every_declared_symbol(lib):
 def test_struct_layouts_match_header():
     # header: 8 int32 + 4 int64 + 2 * 128 int64 + 260 int64
     assert ctypes.sizeof(_native.EclMstStats) == 8 * 4 + 4 * 8 + 2 * 128 * 8 + 260 * 8
-    assert ctypes.sizeof(_native.EclMstOptions) == 6 * 4 + 8
+    assert ctypes.sizeof(_native.EclMstOptions) == 8 * 4 + 8
 
 
 def test_workspace_bytes(lib):
@@ -43,12 +43,13 @@ def test_workspace_bytes(lib):
     assert lib.ecl_mst_workspace_bytes(-1, 10) == 0
     assert lib.ecl_mst_workspace_bytes(10, 1 << 33) == 0
     # C5-sized graph fits comfortably in one B200 (180 GB)
-    assert _native.ecl_mst_workspace_bytes(1 << 26, 2_000_000_000) < 40e9
+    assert _native.ecl_mst_workspace_bytes(1 << 26, 2_000_000_000) < 70e9
 
 
 def test_argument_validation_without_gpu(lib):
     o = _native.default_options()
-    assert o.filter == -1 and o.path_halving == 1 and o.seed == 0x5EED
+    assert o.filter == -1 and o.path_halving == 1 and o.atomic_guards == 1 and o.flatten == 1
+    assert o.seed == 0x5EED
     rc = lib.ecl_mst_device(-1, 0, None, None, None, None, None, None, 0, None, None)
     assert rc == _native.ERR_INVALID
     assert b"negative" in lib.ecl_mst_last_error()
