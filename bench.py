@@ -46,6 +46,7 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-parity", action="store_true")
     ap.add_argument("--flush-mb", type=int, default=512)
+    ap.add_argument("--opt", action="append", default=[], help="ecl_mst_options field=value (ablations)")
     return ap.parse_args()
 
 
@@ -117,23 +118,23 @@ class ClockSampler:
 def algorithmic_bytes(n: int, M: int, st: dict) -> dict:
     """Bytes the method must move per launch.
 
-    init        20 B/vertex  (parent 4 + two key buffers 8+8)
+    init        12 B/vertex  (parent 4 + best-edge key 8)
     populate    8 B/CSR entry (nlist+eweight) + 8 B/vertex (nindex) [+1 B/entry in_mst, phase 1]
                 + per emitted tuple 16 B write + 2x8 B key atomicMin
-                [+ 2x4 B parent gathers per heavy canonical edge, phase 2]
+                [phase 2: + 2x4 B parent gathers per heavy canonical edge, + 8 B/vertex flatten]
     pass A      per input tuple 16 B read + 2x4 B parent; per survivor 16 B write + 2x8 B key min
-    pass B      per tuple 16 B read + 2x8 B key reads; per winner 4 B CAS + 1 B mark + 8 B sum
+    pass B      per tuple 16 B read + 2x8 B key reads; per winner 4 B hook + 8 B key reset + 1 B mark
     """
     live = st["live"]
     win = st["winners"]
     R = len(live)
     p2 = st["phase2_round"]
-    b = {"init": 20 * n}
+    b = {"init": 12 * n}
     b["populate"] = (8 * M + 8 * n + M) + 32 * (live[0] if R else 0)
     passA = passB = 0
     for g in range(1, R):
         if g == p2:
-            b["populate"] += 8 * M + 8 * n + 8 * st["heavy_edges"] + 32 * live[g]
+            b["populate"] += 8 * M + 16 * n + 8 * st["heavy_edges"] + 32 * live[g]
             continue
         passA += 24 * live[g - 1] + 32 * live[g]
     for g in range(R):
@@ -145,7 +146,12 @@ def algorithmic_bytes(n: int, M: int, st: dict) -> dict:
 
 
 def stage_times(st: dict) -> dict:
-    """Split the single kernel's time by the device timestamps (globaltimer)."""
+    """Split the single kernel's time by the device timestamps (globaltimer).
+
+    t_ns[0] start, [1] end of init, [2] end of kernel, [3] end of the
+    flatten step (0 if none), [4+2g] end of pass A / populate of global round
+    g, [5+2g] end of pass B of round g (0 when the round had no pass B).
+    """
     t = st["t_ns"]
     R = st["rounds"]
     if not t or t[0] == 0 or t[2] == 0:
@@ -154,18 +160,28 @@ def stage_times(st: dict) -> dict:
     p2 = st["phase2_round"]
     prev = t[1]
     pop = a = bsum = 0.0
+    flat = 0.0
+    rounds = []
     for g in range(R):
         ta = t[4 + 2 * g]
+        if g == p2 and t[3]:
+            flat = t[3] - prev
+            prev = t[3]
+        da = ta - prev
         if g == 0 or g == p2:
-            pop += ta - prev
+            pop += da
         else:
-            a += ta - prev
+            a += da
         prev = ta
         tb = t[5 + 2 * g]
+        db = 0.0
         if tb and g < R - 1:
-            bsum += tb - prev
+            db = tb - prev
+            bsum += db
             prev = tb
-    out.update(populate_us=pop / 1e3, passA_us=a / 1e3, passB_us=bsum / 1e3, total_us=(t[2] - t[0]) / 1e3)
+        rounds.append([round(da / 1e3, 1), round(db / 1e3, 1)])
+    out.update(populate_us=pop / 1e3, flatten_us=flat / 1e3, passA_us=a / 1e3, passB_us=bsum / 1e3,
+               total_us=(t[2] - t[0]) / 1e3, rounds_AB_us=rounds)
     return out
 
 
@@ -246,10 +262,12 @@ def main():
     total = torch.empty(1, dtype=torch.int64, device=dev)
     flush = torch.empty(args.flush_mb << 20, dtype=torch.uint8, device=dev)
     stream = torch.cuda.current_stream()
+    opt_kw = {k: int(v) for k, v in (o.split("=", 1) for o in args.opt)}
+    opts = eclmst.default_options(**opt_kw)
 
     def step():
         eclmst.ecl_mst_device(n, g.nindex, g.nlist, g.eweight, in_mst_out=in_mst, total_weight_out=total,
-                              workspace=ws, stream=stream)
+                              workspace=ws, options=opts, stream=stream)
 
     for _ in range(max(args.warmup, 3)):
         flush.zero_()
@@ -345,6 +363,7 @@ def main():
         "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
         "config": {"workload": f"{CONFIG_NAMES[args.config]} {g.name}", "n": n, "M": M,
                    "m_undirected": st["canonical_edges"], "parallelism": "replicas" if world > 1 else "single",
+                   "options": opt_kw,
                    "l2": f"inputs ({(8 * M + 8 * n) / 1e6:.0f} MB CSR) exceed L2; plus {args.flush_mb} MB flush "
                          "between steps"},
         "ms_per_graph": ms_max, "ms_per_step_all": per_step, "wall_s": wall,

@@ -63,7 +63,7 @@ typedef struct ecl_mst_options {
     int32_t atomic_guards;   /* 1 (default) load-compare before each atomicMin; 0 always atomic */
     int32_t flatten;         /* 1 (default) compress every path once before the phase-2 populate; 0 off */
     int32_t max_ctas;        /* 0 = fill the GPU (SMs x resident CTAs); else cap the grid */
-    int32_t reserved;
+    int32_t trace;           /* 1: record every CTA's end time of every stage (ecl_mst_read_trace) */
     uint64_t seed;           /* seed of the threshold sample */
 } ecl_mst_options;
 
@@ -123,6 +123,14 @@ int ecl_mst_read_stats(const void *workspace, ecl_mst_stats *stats_out, void *st
  */
 int64_t ecl_mst(int32_t n, const int64_t *nindex, const int32_t *nlist,
                 const int32_t *eweight, uint8_t *in_mst_out);
+
+/* Diagnostics: after a run with opts.trace = 1, synchronises `stream` and
+ * copies the per-CTA stage end times (globaltimer ns) to out[slot * 4096 +
+ * cta] for slot < 2*ECL_MST_MAX_ROUNDS+4 (slot numbering as stats.t_ns) and
+ * cta < stats.grid; at most max_entries values.  Returns ECL_MST_OK or
+ * ECL_MST_ERR_*. */
+#define ECL_MST_TRACE_CTAS 4096
+int ecl_mst_read_trace(const void *workspace, int64_t *out, size_t max_entries, void *stream);
 
 /* Frees the device buffers cached by ecl_mst(). */
 void ecl_mst_release_host_cache(void);

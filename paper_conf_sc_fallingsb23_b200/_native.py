@@ -33,7 +33,7 @@ class EclMstOptions(ctypes.Structure):
         ("atomic_guards", ctypes.c_int32),
         ("flatten", ctypes.c_int32),
         ("max_ctas", ctypes.c_int32),
-        ("reserved", ctypes.c_int32),
+        ("trace", ctypes.c_int32),
         ("seed", ctypes.c_uint64),
     ]
 
@@ -95,6 +95,8 @@ def load(build_if_missing: bool = False):
     L.ecl_mst.restype = i64
     L.ecl_mst.argtypes = [i32, vp, vp, vp, vp]
     L.ecl_mst_release_host_cache.restype = None
+    L.ecl_mst_read_trace.restype = ctypes.c_int
+    L.ecl_mst_read_trace.argtypes = [vp, vp, sz, vp]
     if L.ecl_mst_abi_version() != 1:
         raise ImportError("libeclmst.so ABI version mismatch")
     _lib = L
@@ -103,7 +105,7 @@ def load(build_if_missing: bool = False):
 
 EXPORTED = ["ecl_mst_abi_version", "ecl_mst_last_error", "ecl_mst_default_options",
             "ecl_mst_workspace_bytes", "ecl_mst_device", "ecl_mst_read_stats", "ecl_mst",
-            "ecl_mst_release_host_cache"]
+            "ecl_mst_release_host_cache", "ecl_mst_read_trace"]
 
 
 def _err(code):
@@ -199,6 +201,20 @@ def ecl_mst_read_stats(workspace, stream=None) -> dict:
         "live": list(st.live[:R]), "winners": list(st.winners[:R]),
         "t_ns": list(st.t_ns[: 2 * R + 4]),
     }
+
+
+TRACE_CTAS = 4096
+
+
+def ecl_mst_read_trace(workspace, stats, stream=None):
+    """Per-CTA stage end times of the last traced run: int64 [slots, grid] (ns)."""
+    slots = 2 * MAX_ROUNDS + 4
+    out = torch.zeros(slots * TRACE_CTAS, dtype=torch.int64)
+    with torch.cuda.device(workspace.device):
+        rc = load().ecl_mst_read_trace(workspace.data_ptr(), out.data_ptr(), out.numel(), _stream_ptr(stream))
+    if rc != OK:
+        _err(rc)
+    return out.view(slots, TRACE_CTAS)[:, : stats["grid"]]
 
 
 def ecl_mst(n, nindex, nlist, eweight, in_mst_out):

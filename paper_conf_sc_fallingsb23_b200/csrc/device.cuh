@@ -33,11 +33,14 @@ __device__ __forceinline__ unsigned long long globaltimer_ns() {
 }
 
 // ---------------------------------------------------------------------------
-// disjoint sets.  parent[] is read through L2 (ld.global.cg): other SMs write
-// it (hooks in pass B, halving anywhere) and L1 is not coherent.  Every
-// parent pointer forms a forest (a vertex is only ever re-pointed to one of
-// its ancestors, or -- a root, once -- to a vertex of another set), so every
-// walk terminates.
+// disjoint sets.  Within one stage of the persistent kernel parent[] only
+// changes by path halving (a vertex re-pointed to one of its ancestors) or,
+// in pass B, by hooking roots -- and pass B never reads it.  Every grid
+// barrier ends with a gpu-scope fence, which invalidates L1 (CCTL.IVALL), so a
+// find() may read parent[] through L1 (ld.global.ca): a stale cached pointer
+// is still an ancestor, and roots cannot change while finds run.  Hot roots
+// (one giant set touched by millions of edges) are then served by L1 instead
+// of one L2 slice.
 // ---------------------------------------------------------------------------
 
 // Continue a find() from x whose parent px is already loaded.  With halving
@@ -45,23 +48,25 @@ __device__ __forceinline__ unsigned long long globaltimer_ns() {
 // a benign race: the stored value is always an ancestor).
 __device__ __forceinline__ int find_from(int* __restrict__ parent, int x, int px, bool halving) {
     while (px != x) {
-        const int ppx = __ldcg(parent + px);
+        const int ppx = __ldca(parent + px);
         if (ppx == px) return px;
-        if (halving) __stcg(parent + x, ppx);
+        if (halving) parent[x] = ppx;
         x = ppx;
-        px = __ldcg(parent + x);
+        px = __ldca(parent + x);
     }
     return x;
 }
 
 __device__ __forceinline__ int find_root(int* __restrict__ parent, int x, bool halving) {
-    return find_from(parent, x, __ldcg(parent + x), halving);
+    return find_from(parent, x, __ldca(parent + x), halving);
 }
 
 // 64-bit atomicMin (L20-21) with the paper's optional guard: a plain
-// L2 load first, skipping the atomic when it cannot lower the slot.
+// load first, skipping the atomic when it cannot lower the slot.  The guard
+// may read through L1: slots only decrease during a pass, so a stale value is
+// >= the current one and a skipped atomic could never have lowered the slot.
 __device__ __forceinline__ void record_min(long long* slot, long long key, bool guard) {
-    if (!guard || __ldcg(slot) > key) atomicMin(slot, key);
+    if (!guard || __ldca(slot) > key) atomicMin(slot, key);
 }
 
 // Warp-level compaction of one chunk (kItems tuples per lane, any order):

@@ -57,8 +57,11 @@ struct Internal {
     unsigned int pad[63];
 };
 
+constexpr int kTraceSlots = 2 * ECL_MST_MAX_ROUNDS + 4;
+static_assert(kMaxGrid == ECL_MST_TRACE_CTAS, "trace layout");
+
 struct Layout {
-    size_t stats, internal, key, parent, wl0, wl1, total;
+    size_t stats, internal, trace, key, parent, wl0, wl1, total;
 };
 
 static inline size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
@@ -68,6 +71,7 @@ static inline Layout layout_for(int64_t n, int64_t M) {
     size_t off = 0;
     L.stats = off;    off = align_up(off + sizeof(ecl_mst_stats), 256);
     L.internal = off; off = align_up(off + sizeof(Internal), 256);
+    L.trace = off;    off = align_up(off + sizeof(long long) * kTraceSlots * kMaxGrid, 256);
     L.key = off;      off = align_up(off + sizeof(long long) * (size_t)n, 256);
     L.parent = off;   off = align_up(off + sizeof(int) * (size_t)n, 256);
     L.wl0 = off;      off = align_up(off + sizeof(int4) * (size_t)M, 256);
@@ -87,6 +91,7 @@ struct Params {
     long long* total_out;
     ecl_mst_stats* st;
     Internal* in;
+    long long* trace;                 // [kTraceSlots][kMaxGrid] or null
     long long* key;
     int* parent;
     int4* wl0;
@@ -129,16 +134,14 @@ __device__ __forceinline__ void populate(const Params& P, long long wb, long lon
     const bool halving = P.halving != 0, guard = P.guards != 0;
     long long* __restrict__ K = P.key;
     int r_cur = r_first;
-    for (long long c0 = wb; c0 < we; c0 += kChunk) {
+    // software pipeline: the next chunk's CSR entries are in flight while the
+    // current chunk searches rows, records keys and emits tuples
+    int nv[kItems], nw[kItems];
+    auto load_chunk = [&](long long c0, int (&vv)[kItems], int (&ww)[kItems]) {
         const long long c1 = min(c0 + (long long)kChunk, we);
         const int len = (int)(c1 - c0);
-        const bool need_carry = c1 < we;
         const int p0 = lane * kItems;
-        const bool full = p0 + kItems <= len;
-
-        // stream the chunk's entries first (independent of the row search)
-        int vv[kItems], ww[kItems];
-        if (P.vec_ok && full) {
+        if (P.vec_ok && p0 + kItems <= len) {
             const int4 a = __ldcs(reinterpret_cast<const int4*>(P.nlist + c0 + p0));
             const int4 b = __ldcs(reinterpret_cast<const int4*>(P.eweight + c0 + p0));
             vv[0] = a.x; vv[1] = a.y; vv[2] = a.z; vv[3] = a.w;
@@ -151,6 +154,21 @@ __device__ __forceinline__ void populate(const Params& P, long long wb, long lon
                 ww[k] = ok ? __ldcs(P.eweight + c0 + p0 + k) : 0;
             }
         }
+    };
+    if (wb < we) load_chunk(wb, nv, nw);
+    for (long long c0 = wb; c0 < we; c0 += kChunk) {
+        const long long c1 = min(c0 + (long long)kChunk, we);
+        const int len = (int)(c1 - c0);
+        const bool need_carry = c1 < we;
+        const int p0 = lane * kItems;
+        const bool full = p0 + kItems <= len;
+        int vv[kItems], ww[kItems];
+#pragma unroll
+        for (int k = 0; k < kItems; ++k) {
+            vv[k] = nv[k];
+            ww[k] = nw[k];
+        }
+        if (c1 < we) load_chunk(c1, nv, nw);
 
         // row of every entry: mark row starts inside the chunk, then max-scan
 #pragma unroll
@@ -263,8 +281,8 @@ __device__ __forceinline__ void passA(const Params& P, const int4* __restrict__ 
 #pragma unroll
         for (int i = 0; i < kItems; ++i) {
             if (keep[i]) {
-                px[i] = __ldcg(parent + t[i].x);
-                qx[i] = __ldcg(parent + t[i].y);
+                px[i] = __ldca(parent + t[i].x);
+                qx[i] = __ldca(parent + t[i].y);
             }
         }
 #pragma unroll
@@ -304,19 +322,23 @@ __device__ __forceinline__ void passB(const Params& P, const int4* __restrict__ 
             ok[i] = idx < cnt;
             t[i] = ok[i] ? __ldcg(wl + idx) : make_int4(0, 0, 0, 0);
         }
-        long long kp[kItems], kq[kItems];
+        // Only the id half of each slot is compared: ids are unique per
+        // edge, so id equality is key equality (and inf's id half, 2^32-1,
+        // is never a valid id).  L1 is fine: K[p] only changes when p's own
+        // winner resets it.
+        const unsigned* __restrict__ Kid = reinterpret_cast<const unsigned*>(K);
+        unsigned kp[kItems], kq[kItems];
 #pragma unroll
         for (int i = 0; i < kItems; ++i) {
             if (ok[i]) {
-                kp[i] = __ldcg(K + t[i].x);
-                kq[i] = __ldcg(K + t[i].y);
+                kp[i] = __ldca(Kid + 2 * (long long)t[i].x);
+                kq[i] = __ldca(Kid + 2 * (long long)t[i].y);
             }
         }
 #pragma unroll
         for (int i = 0; i < kItems; ++i) {
             if (!ok[i]) continue;
-            const long long key = make_key(t[i].z, (unsigned)t[i].w);
-            const bool wp = kp[i] == key, wq = kq[i] == key;          // L29
+            const bool wp = kp[i] == (unsigned)t[i].w, wq = kq[i] == (unsigned)t[i].w;   // L29
             if (wp || wq) {
                 const int p = t[i].x, q = t[i].y;
                 // L30 join: each set hooks along its own lightest edge;
@@ -330,6 +352,14 @@ __device__ __forceinline__ void passB(const Params& P, const int4* __restrict__ 
                 wcnt += 1;
             }
         }
+    }
+}
+
+// per-CTA end of a stage (diagnostics; P.trace is null unless opts.trace)
+__device__ __forceinline__ void trace_cta(const Params& P, int slot) {
+    if (P.trace && slot < kTraceSlots) {
+        __syncthreads();
+        if (threadIdx.x == 0) P.trace[(long long)slot * kMaxGrid + blockIdx.x] = (long long)globaltimer_ns();
     }
 }
 
@@ -396,6 +426,7 @@ __global__ void __launch_bounds__(kBlock, 2) mst_persistent(Params P) {
         }
         if (tid == 0) P.in->done = 0u;
     }
+    trace_cta(P, 1);
     grid.sync();
     const bool filtered = __ldcg(&st->filtered) != 0;
     const int T = __ldcg(&st->threshold);
@@ -415,9 +446,11 @@ __global__ void __launch_bounds__(kBlock, 2) mst_persistent(Params P) {
             if (P.flatten) {   // compress every path once: phase-2 finds become one hop
                 for (long long v = (long long)blockIdx.x * kBlock + tid; v < P.n; v += (long long)gridDim.x * kBlock) {
                     const int r = find_root(P.parent, (int)v, true);
-                    if (r != (int)v) __stcg(P.parent + v, r);
+                    if (r != (int)v) P.parent[v] = r;
                 }
+                trace_cta(P, 3);
                 grid.sync();
+                stamp(P, 3);
             }
             ++g;
             if (b0 && tid == 0) st->phase2_round = g;
@@ -436,6 +469,7 @@ __global__ void __launch_bounds__(kBlock, 2) mst_persistent(Params P) {
             if (lane == 0 && c) atomicAdd(reinterpret_cast<unsigned long long*>(&st->canonical_edges), (unsigned long long)c);
             if (lane == 0 && h) atomicAdd(reinterpret_cast<unsigned long long*>(&st->heavy_edges), (unsigned long long)h);
         }
+        trace_cta(P, 4 + 2 * g);
         grid.sync();
         stamp(P, 4 + 2 * g);
         long long L = __ldcg(&st->live[g]);
@@ -445,6 +479,7 @@ __global__ void __launch_bounds__(kBlock, 2) mst_persistent(Params P) {
             const long long d = warp_sum(wcnt - w0);
             if (lane == 0 && d) atomicAdd(reinterpret_cast<unsigned long long*>(&st->winners[g]), (unsigned long long)d);
             if (tid == 0) s_out = 0;
+            trace_cta(P, 5 + 2 * g);
             grid.sync();
             stamp(P, 5 + 2 * g);
             if (g + 1 >= ECL_MST_MAX_ROUNDS) { overflow = true; break; }
@@ -454,6 +489,7 @@ __global__ void __launch_bounds__(kBlock, 2) mst_persistent(Params P) {
             __syncthreads();
             cnt = s_out;
             if (tid == 0 && cnt) atomicAdd(reinterpret_cast<unsigned long long*>(&st->live[g]), (unsigned long long)cnt);
+            trace_cta(P, 4 + 2 * g);
             grid.sync();
             stamp(P, 4 + 2 * g);
             L = __ldcg(&st->live[g]);
@@ -550,6 +586,7 @@ void ecl_mst_default_options(ecl_mst_options* o) {
     o->atomic_guards = 1;
     o->flatten = 1;
     o->max_ctas = 0;
+    o->trace = 0;
     o->seed = 0x5eedull;
 }
 
@@ -614,6 +651,7 @@ int ecl_mst_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t* n
     P.total_out = reinterpret_cast<long long*>(total_weight_out);
     P.st = reinterpret_cast<ecl_mst_stats*>(ws + L.stats);
     P.in = reinterpret_cast<Internal*>(ws + L.internal);
+    P.trace = o.trace ? reinterpret_cast<long long*>(ws + L.trace) : nullptr;
     P.key = reinterpret_cast<long long*>(ws + L.key);
     P.parent = reinterpret_cast<int*>(ws + L.parent);
     P.wl0 = reinterpret_cast<int4*>(ws + L.wl0);
@@ -641,6 +679,20 @@ int ecl_mst_read_stats(const void* workspace, ecl_mst_stats* out, void* stream) 
     cudaError_t e = cudaMemcpyAsync(out, workspace, sizeof(ecl_mst_stats), cudaMemcpyDeviceToHost, s);
     if (e == cudaSuccess) e = cudaStreamSynchronize(s);
     if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "read_stats: %s", cudaGetErrorString(e));
+    return ECL_MST_OK;
+}
+
+int ecl_mst_read_trace(const void* workspace, int64_t* out, size_t max_entries, void* stream) {
+    g_last_error.clear();
+    if (!workspace || !out) return fail(ECL_MST_ERR_INVALID, "null argument");
+    const Layout L = layout_for(0, 0);
+    size_t count = (size_t)kTraceSlots * kMaxGrid;
+    if (count > max_entries) count = max_entries;
+    cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+    cudaError_t e = cudaMemcpyAsync(out, static_cast<const char*>(workspace) + L.trace, count * sizeof(int64_t),
+                                    cudaMemcpyDeviceToHost, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "read_trace: %s", cudaGetErrorString(e));
     return ECL_MST_OK;
 }
 

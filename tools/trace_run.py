@@ -1,0 +1,71 @@
+"""Per-CTA stage timing of the persistent kernel (load imbalance diagnostics).
+
+  python tools/trace_run.py --config rmat [--opt atomic_guards=0 ...]
+
+For every stage (populate / pass A / pass B of each global round) prints the
+stage duration (last CTA done - previous barrier) and how early the typical
+and the first CTA finished: a large gap means CTAs wait at the grid barrier.
+"""
+import argparse
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+import torch  # noqa: E402
+
+import paper_conf_sc_fallingsb23_b200 as eclmst  # noqa: E402
+import synth  # noqa: E402
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--config", default="road")
+    ap.add_argument("--size", default="full")
+    ap.add_argument("--opt", action="append", default=[])
+    ap.add_argument("--runs", type=int, default=3)
+    args = ap.parse_args()
+    dev = torch.device("cuda:0")
+    g = synth.make_config(args.config, args.size, device=dev)
+    kw = {k: int(v) for k, v in (o.split("=") for o in args.opt)}
+    kw["trace"] = 1
+    opts = eclmst.default_options(**kw)
+    ws = torch.empty(eclmst.ecl_mst_workspace_bytes(g.n, g.M), dtype=torch.uint8, device=dev)
+    for _ in range(args.runs):
+        eclmst.ecl_mst_device(g.n, g.nindex, g.nlist, g.eweight, workspace=ws, options=opts)
+    st = eclmst.ecl_mst_read_stats(ws)
+    tr = eclmst.ecl_mst_read_trace(ws, st).double()
+    t = st["t_ns"]
+    print(f"{g.name} opts={kw} total {(t[2] - t[0]) / 1e3:.1f} us  rounds {st['rounds']} grid {st['grid']}")
+    prev = t[1]
+    R, p2 = st["rounds"], st["phase2_round"]
+    seq = []
+    for r in range(R):
+        if r == p2 and t[3]:
+            seq.append(("flatten", 3))
+        seq.append(("populate" if r in (0, p2) else "passA", 4 + 2 * r, r))
+        if r < R - 1 and t[5 + 2 * r]:
+            seq.append(("passB", 5 + 2 * r, r))
+    tot_wait = 0.0
+    for item in seq:
+        name, slot = item[0], item[1]
+        r = item[2] if len(item) > 2 else -1
+        row = tr[slot]
+        valid = row[row > 0]
+        if valid.numel() == 0:
+            continue
+        end = t[slot] if t[slot] else float(valid.max())
+        dur = (float(valid.max()) - prev) / 1e3
+        med = (float(valid.median()) - prev) / 1e3
+        mn = (float(valid.min()) - prev) / 1e3
+        wait = float((valid.max() - valid).mean()) / 1e3
+        tot_wait += wait
+        live = st["live"][r] if r >= 0 else 0
+        print(f"  r{r:<3d} {name:9s} live {live:>11d}  last {dur:8.1f} us  median {med:8.1f}  first {mn:8.1f}  "
+              f"mean wait {wait:7.1f}")
+        prev = end
+    print(f"  sum of mean CTA wait at barriers: {tot_wait:.1f} us")
+
+
+if __name__ == "__main__":
+    main()
