@@ -24,6 +24,8 @@
  *   nindex   int64[n+1], nindex[0] = 0, non-decreasing, nindex[n] = M.
  *   nlist    int32[M], 0 <= nlist[j] < n: the neighbour of entry j.
  *   eweight  int32[M]: the weight of entry j (any int32 value).
+ *            (device call: nlist and eweight 16-byte aligned, in_mst 4-byte
+ *            aligned -- any cudaMalloc/torch allocation is)
  *   in_mst   uint8[M] OUTPUT: 1 iff entry j is the id of an MSF edge, else 0
  *            (mirror slots are always 0).  Every byte is written.
  * Ownership: the caller owns every buffer; inputs are only read.  The library
@@ -60,7 +62,9 @@ typedef struct ecl_mst_options {
     int32_t threshold_mode;  /* 0 sampled: 20 weights, c = 4 (reading Q5/Q7); 1 fixed */
     int32_t threshold;       /* phase 1 takes w < threshold when threshold_mode == 1 */
     int32_t path_halving;    /* 1 (default) find() halves paths it walks (P:142 reading Q15); 0 off */
-    int32_t atomic_guards;   /* 1 (default) load-compare before each atomicMin; 0 always atomic */
+    int32_t atomic_guards;   /* load-compare before each atomicMin: 1 everywhere; 0 never;
+                                -1 (default) everywhere except the phase-1 populate, where the
+                                slots are still mostly inf and the guard only adds latency */
     int32_t flatten;         /* 1 (default) compress every path once before the phase-2 populate; 0 off */
     int32_t max_ctas;        /* 0 = fill the GPU (SMs x resident CTAs); else cap the grid */
     int32_t trace;           /* 1: record every CTA's end time of every stage (ecl_mst_read_trace) */
@@ -86,19 +90,21 @@ typedef struct ecl_mst_stats {
     int64_t t_ns[2 * ECL_MST_MAX_ROUNDS + 4]; /* device timestamps (globaltimer) per stage */
 } ecl_mst_stats;
 
-/* Default options (filter auto, sampled threshold, seed 0x5eed, halving,
- * guards and flatten on). */
+/* Default options (filter auto, sampled threshold, seed 0x5eed, halving and
+ * flatten on, guards auto). */
 void ecl_mst_default_options(ecl_mst_options *opts);
 
 /* Bytes of device workspace ecl_mst_device needs for (n, M); 0 if too large.
- * Layout: header+stats, key[n] int64 (best-edge
- * slots), parent[n] int32, two worklists int4[M] (in / out of a pass). */
+ * Layout: header+stats, per-arena counters, trace,
+ * chunk start rows int32[M/128], key[n] int64 (best-edge slots), parent[n]
+ * int32, two worklists int4[~M] (in / out of a pass). */
 size_t ecl_mst_workspace_bytes(int64_t n, int64_t M);
 
 /*
  * The hot path.  All pointers are DEVICE pointers (current device).  Runs
  * asynchronously on `stream` (a cudaStream_t; NULL = legacy default stream)
- * as ONE persistent cooperative kernel: no host round-trips per round.
+ * as a fixed sequence of kernels whose round loop is one persistent
+ * cooperative kernel per phase: no host round-trips.
  * total_weight_out (device int64*) receives the MSF weight, or INT64_MIN if
  * the device detected an inconsistent CSR (then stats.status = ERR_INPUT and
  * in_mst is unspecified).  workspace must be >= ecl_mst_workspace_bytes(n, M)

@@ -1,37 +1,35 @@
 // ecl_mst.cu -- B200 (sm_100a) implementation of the ECL-MST hot path behind
 // the C ABI in include/ecl_mst.h.
 //
-// One persistent cooperative kernel per MSF (no host round-trips per round,
-// replacing the paper's host while-loop with a cudaMemcpy per iteration,
-// P:86-88).  Grid = SMs x resident CTAs; every warp owns a contiguous
-// range of CSR entries, every CTA the union of its warps' ranges and the same
-// slice of the two worklists.  Warps work independently (warp-level
-// compaction, no CTA barriers inside a pass); stages are separated by grid
-// barriers:
+// One MSF = one stream-ordered sequence of kernels, no host round-trip:
 //
-//   init      Alg. 1: parent[v] = v, key[v] = inf; block 0 draws the
-//             filter threshold; each warp finds the row of its
-//             first CSR entry.
-//   populate  Alg. 2 L1-11 over the warp's CSR range (edge-balanced), FUSED
-//             with round 0 of L14-21 (all endpoints are roots then, so the
-//             find is the identity and nothing is dropped): emit <u,v,w,id>
-//             for u < v (L4) meeting the threshold (L6), atomicMin the key
-//             into both endpoints.  Phase 2 re-reads the CSR for the
-//             heavy edges, replaces endpoints by set(u), set(v), drops
-//             intra-set edges (the filter) and records keys the same way.
-//   pass B    L27-31: an edge whose key won at endpoint p hooks p under the
-//             other endpoint (Boruvka hooking: each representative is written
-//             by exactly one edge, so no CAS is needed; a mutual pair keeps
-//             its smaller end as root), marks in_mst[id] and adds its weight.
-//             The winning edge of p also resets key[p] (L34-37 fused: an edge
-//             that lost at p compares unequal to both the old minimum and to
-//             inf, so the early reset cannot change any decision).
-//   pass A    L14-23 of the next round: find (implicit path compression,
-//             L15-18), drop p == q, keep <p,q,w,id> in the other worklist,
-//             atomicMin the key into both representatives.
-//   flatten   before phase 2: parent[v] = find(v) for every v.
-//
-// Loop per phase: populate ; while (live > 0) { B ; A }.
+//   k_init        Alg. 1: parent[v] = v, key[v] = inf; chunk start
+//                 rows (so populate needs no search); block 0 draws the filter
+//                 threshold and checks nindex.
+//   k_populate<1> Alg. 2 L1-11 fused with round 0 of L14-21: one warp per
+//                 128-entry CSR chunk (edge-centric, high occupancy).  Emits
+//                 <u,v,w,id> for u < v (L4) meeting the threshold (L6) into
+//                 one of G arenas (round-robin by CTA, so every arena samples
+//                 the whole CSR evenly) and atomicMins the key into both
+//                 endpoints (all endpoints are roots in round 0).
+//   k_rounds      persistent cooperative kernel, CTA b owns arena b:
+//                 while (live > 0) { pass B ; pass A } with grid barriers.
+//                 pass B  L27-31: an edge whose key won at endpoint p hooks p
+//                         under the other endpoint (Boruvka hooking: each
+//                         representative is written by exactly one edge, no
+//                         CAS; a mutual pair keeps its smaller end as root),
+//                         marks in_mst[id], adds its weight, and resets
+//                         key[p] (L34-37 fused: an edge that lost at p compares
+//                         unequal to the old minimum and to inf alike).
+//                 pass A  L14-23: find (implicit path compression L15-18),
+//                         drop p == q, compact <p,q,w,id> into the other
+//                         worklist, atomicMin the key into both sets.
+//   k_flatten     phase 2 only: parent[v] = find(v), so every vertex points
+//                 at its root.
+//   k_populate<2> P:152: heavy edges, endpoints replaced by set(u), set(v)
+//                 (one load each after flattening), intra-set edges filtered.
+//   k_rounds      phase 2 rounds (exits at once when there is no phase 2).
+//   k_finalize    total weight / status -> caller's output.
 #include <cooperative_groups.h>
 #include <cuda_runtime.h>
 
@@ -40,6 +38,7 @@
 #include <cstdint>
 #include <cstdio>
 #include <cstring>
+#include <algorithm>
 #include <mutex>
 #include <string>
 
@@ -50,32 +49,52 @@ namespace cg = cooperative_groups;
 
 namespace eclmst {
 
-constexpr int kMaxGrid = 4096;
-
-struct Internal {
-    unsigned int done;      // end-of-kernel ticket
-    unsigned int pad[63];
-};
-
+constexpr int kMaxGrid = 4096;                 // CTAs of k_rounds (= arenas), upper bound
+constexpr int kPopWarps = 8;                   // warps per k_populate CTA (one chunk each)
+constexpr int kPopBlock = 32 * kPopWarps;
 constexpr int kTraceSlots = 2 * ECL_MST_MAX_ROUNDS + 4;
 static_assert(kMaxGrid == ECL_MST_TRACE_CTAS, "trace layout");
 
+struct Internal {
+    unsigned int done;                 // unused ticket
+    int g_cur;                         // first global round of the running phase
+    int g_end;                         // last global round of the finished phase
+    int pad0;
+    int arena_cnt[kMaxGrid];           // tuples emitted into each arena by k_populate
+    long long arena_canon[kMaxGrid];   // canonical edges seen, per arena (phase 1)
+    long long arena_heavy[kMaxGrid];   // heavy canonical edges, per arena (phase 1)
+};
+
 struct Layout {
-    size_t stats, internal, trace, key, parent, wl0, wl1, total;
+    size_t stats, internal, trace, rowstart, key, parent, wl0, wl1, total;
+    long long wl_cap;                  // tuples per worklist buffer
 };
 
 static inline size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
 
+static inline long long ceil_div(long long a, long long b) { return (a + b - 1) / b; }
+
+// worklist tuples needed for G arenas of ceil(nchunks/G)*kChunk tuples, for
+// any G <= min(kMaxGrid, nchunks)
+static inline long long wl_capacity(long long M) {
+    const long long nchunks = ceil_div(M, kChunk);
+    const long long gmax = nchunks < kMaxGrid ? nchunks : kMaxGrid;
+    return (nchunks + gmax) * (long long)kChunk;
+}
+
 static inline Layout layout_for(int64_t n, int64_t M) {
     Layout L;
     size_t off = 0;
+    const long long nchunks = ceil_div(M, kChunk);
+    L.wl_cap = wl_capacity(M);
     L.stats = off;    off = align_up(off + sizeof(ecl_mst_stats), 256);
     L.internal = off; off = align_up(off + sizeof(Internal), 256);
     L.trace = off;    off = align_up(off + sizeof(long long) * kTraceSlots * kMaxGrid, 256);
+    L.rowstart = off; off = align_up(off + sizeof(int) * (size_t)(nchunks + 1), 256);
     L.key = off;      off = align_up(off + sizeof(long long) * (size_t)n, 256);
     L.parent = off;   off = align_up(off + sizeof(int) * (size_t)n, 256);
-    L.wl0 = off;      off = align_up(off + sizeof(int4) * (size_t)M, 256);
-    L.wl1 = off;      off = align_up(off + sizeof(int4) * (size_t)M, 256);
+    L.wl0 = off;      off = align_up(off + sizeof(int4) * (size_t)L.wl_cap, 256);
+    L.wl1 = off;      off = align_up(off + sizeof(int4) * (size_t)L.wl_cap, 256);
     L.total = off;
     return L;
 }
@@ -83,7 +102,9 @@ static inline Layout layout_for(int64_t n, int64_t M) {
 struct Params {
     int n;
     long long M;
-    long long sub;                    // CSR entries per warp (multiple of kItems)
+    long long nchunks;                // ceil(M / kChunk)
+    int G;                            // k_rounds CTAs = arenas
+    long long cap;                    // tuples per arena
     const long long* __restrict__ nindex;
     const int* __restrict__ nlist;
     const int* __restrict__ eweight;
@@ -92,6 +113,7 @@ struct Params {
     ecl_mst_stats* st;
     Internal* in;
     long long* trace;                 // [kTraceSlots][kMaxGrid] or null
+    int* rowstart;                    // row of CSR entry c*kChunk, per chunk
     long long* key;
     int* parent;
     int4* wl0;
@@ -101,47 +123,133 @@ struct Params {
     int threshold_mode;
     int threshold_value;
     int halving;
-    int guards;
+    int guards;                       // -1 auto, 0 off, 1 on
     int flatten;
-    int vec_ok;
 };
 
-// inclusive max-scan over a warp's chunk (kItems consecutive values per lane)
-__device__ __forceinline__ void warp_max_scan(int (&m)[kItems]) {
-    const int lane = threadIdx.x & 31;
-#pragma unroll
-    for (int k = 1; k < kItems; ++k) m[k] = max(m[k], m[k - 1]);
-    int incl = m[kItems - 1];
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        const int y = __shfl_up_sync(kFull, incl, o);
-        if (lane >= o) incl = max(incl, y);
-    }
-    int excl = __shfl_up_sync(kFull, incl, 1);
-    if (lane == 0) excl = INT_MIN;
-#pragma unroll
-    for (int k = 0; k < kItems; ++k) m[k] = max(m[k], excl);
+__device__ __forceinline__ void stamp(const Params& P, int slot) {
+    if (blockIdx.x == 0 && threadIdx.x == 0 && slot < kTraceSlots)
+        P.st->t_ns[slot] = (long long)globaltimer_ns();
 }
 
-// Alg. 2 L1-11 (+ round 0 of L14-21) over one warp's CSR range [wb, we).
-// PH = 1: light edges; PH = 2: heavy edges with set() endpoints and the
-// cycle filter.
+// per-CTA end of a stage (diagnostics; P.trace is null unless opts.trace)
+__device__ __forceinline__ void trace_cta(const Params& P, int slot) {
+    if (P.trace && slot < kTraceSlots) {
+        __syncthreads();
+        if (threadIdx.x == 0) P.trace[(long long)slot * kMaxGrid + blockIdx.x] = (long long)globaltimer_ns();
+    }
+}
+
+// phase 2 runs iff filtering is on and phase 1 deferred at least one edge
+__device__ __forceinline__ bool phase2_needed(const Params& P) {
+    return __ldcg(&P.st->filtered) != 0 && __ldcg(&P.st->heavy_edges) != 0;
+}
+
+// ---------------------------------------------------------------------------
+// k_init: Alg. 1 + chunk start rows + threshold
+// ---------------------------------------------------------------------------
+__global__ void __launch_bounds__(256) k_init(Params P) {
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const long long stride = (long long)gridDim.x * blockDim.x;
+    const long long i0 = (long long)blockIdx.x * blockDim.x + tid;
+    bool err = false;
+    for (long long v = i0; v < P.n; v += stride) {
+        P.parent[v] = (int)v;                       // every vertex its own set
+        P.key[v] = kInf;                            // no minimum edge recorded
+        // chunk starts inside row v: rowstart[c] = v for c*kChunk in [s, e)
+        const long long s = P.nindex[v], e = P.nindex[v + 1];
+        if (e < s) err = true;
+        for (long long c = (s + kChunk - 1) / kChunk; c * kChunk < e && c < P.nchunks; ++c) P.rowstart[c] = (int)v;
+    }
+    if (blockIdx.x == 0) {
+        ecl_mst_stats* st = P.st;   // zeroed by a memset node just before this kernel
+        for (int i = tid; i < P.G; i += blockDim.x) {
+            P.in->arena_cnt[i] = 0;
+            P.in->arena_canon[i] = 0;
+            P.in->arena_heavy[i] = 0;
+        }
+        __syncthreads();
+        if (warp == 0) {
+            // filter decision (P:143-145, P:152; readings Q5-Q7)
+            const bool filtered = P.filter_mode < 0 ? (P.M >= 4LL * P.n) : (P.filter_mode != 0);
+            int T = INT_MAX;
+            if (filtered) {
+                if (P.threshold_mode == 1) {
+                    T = P.threshold_value;
+                } else {
+                    int w = INT_MAX;
+                    if (lane < 20) {
+                        const unsigned long long h = splitmix64(P.seed * 0x100000001B3ull + (unsigned long long)lane);
+                        w = P.eweight[(long long)(h % (unsigned long long)P.M)];
+                    }
+                    int rank = 0;
+                    for (int s = 0; s < 20; ++s) {
+                        const int ws = __shfl_sync(kFull, w, s);
+                        if (lane < 20 && (ws < w || (ws == w && s < lane))) ++rank;
+                    }
+                    long long kpos = (80LL * P.n) / P.M;   // c|V| lightest of M entries: 20 * 4n / M
+                    if (kpos > 19) kpos = 19;
+                    const unsigned b = __ballot_sync(kFull, lane < 20 && rank == (int)kpos);
+                    T = __shfl_sync(kFull, w, __ffs(b) - 1);
+                }
+            }
+            if (lane == 0) {
+                st->t_ns[0] = (long long)globaltimer_ns();
+                st->filtered = filtered ? 1 : 0;
+                st->threshold = T;
+                st->grid = P.G;
+                st->block = kBlock;
+                st->phase2_round = -1;
+                if (P.nindex[0] != 0 || P.nindex[P.n] != P.M) err = true;
+                P.in->g_cur = 0;
+                P.in->g_end = 0;
+                P.in->done = 0;
+            }
+        }
+    }
+    if (err) atomicExch(&P.st->status, ECL_MST_ERR_INPUT);
+}
+
+// ---------------------------------------------------------------------------
+// k_populate<PH>: one warp per 128-entry CSR chunk
+// ---------------------------------------------------------------------------
 template <int PH>
-__device__ __forceinline__ void populate(const Params& P, long long wb, long long we, int r_first,
-                                         bool filtered, int T, int* s_mark, int4* __restrict__ out, int* s_out,
-                                         long long& canon_cnt, long long& heavy_cnt, int& err) {
-    const int lane = threadIdx.x & 31;
-    const bool halving = P.halving != 0, guard = P.guards != 0;
+__global__ void __launch_bounds__(kPopBlock, 8) k_populate(Params P) {
+    __shared__ int s_mark[kPopWarps][kChunk];
+    __shared__ long long s_canon[kPopWarps], s_heavy[kPopWarps];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    if (PH == 2 && !phase2_needed(P)) return;
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        if (PH == 1) P.st->t_ns[1] = (long long)globaltimer_ns();   // init done
+        else P.st->t_ns[3] = (long long)globaltimer_ns();           // flatten done
+    }
+    const bool filtered = __ldcg(&P.st->filtered) != 0;
+    const int T = __ldcg(&P.st->threshold);
+    const bool guard = (P.guards > 0) || (P.guards < 0 && PH == 2);
     long long* __restrict__ K = P.key;
-    int r_cur = r_first;
-    // software pipeline: the next chunk's CSR entries are in flight while the
-    // current chunk searches rows, records keys and emits tuples
-    int nv[kItems], nw[kItems];
-    auto load_chunk = [&](long long c0, int (&vv)[kItems], int (&ww)[kItems]) {
-        const long long c1 = min(c0 + (long long)kChunk, we);
+    const long long c = (long long)blockIdx.x * kPopWarps + warp;
+    // chunk-level round robin over the arenas: every arena samples the whole
+    // CSR, so the round kernel's CTAs start with balanced work even where
+    // the density of u < v entries drifts along the rows
+    const int arena = (int)(c % P.G);
+    int4* out = P.wl0 + (long long)arena * P.cap;
+    bool keep[kItems];
+    int4 t[kItems];
+    long long canon_cnt = 0, heavy_cnt = 0;
+    bool err = false;
+#pragma unroll
+    for (int k = 0; k < kItems; ++k) keep[k] = false;
+
+    if (c < P.nchunks) {
+        const long long c0 = c * kChunk;
+        const long long c1 = min(c0 + (long long)kChunk, P.M);
         const int len = (int)(c1 - c0);
         const int p0 = lane * kItems;
-        if (P.vec_ok && p0 + kItems <= len) {
+        // rows of this chunk: r0 = row of entry c0; rows r0+1 .. r_last start inside
+        const int r0 = P.rowstart[c];
+        const int r_last = (c + 1 < P.nchunks) ? P.rowstart[c + 1] : P.n - 1;
+        int vv[kItems], ww[kItems];
+        if (p0 + kItems <= len) {
             const int4 a = __ldcs(reinterpret_cast<const int4*>(P.nlist + c0 + p0));
             const int4 b = __ldcs(reinterpret_cast<const int4*>(P.eweight + c0 + p0));
             vv[0] = a.x; vv[1] = a.y; vv[2] = a.z; vv[3] = a.w;
@@ -154,53 +262,38 @@ __device__ __forceinline__ void populate(const Params& P, long long wb, long lon
                 ww[k] = ok ? __ldcs(P.eweight + c0 + p0 + k) : 0;
             }
         }
-    };
-    if (wb < we) load_chunk(wb, nv, nw);
-    for (long long c0 = wb; c0 < we; c0 += kChunk) {
-        const long long c1 = min(c0 + (long long)kChunk, we);
-        const int len = (int)(c1 - c0);
-        const bool need_carry = c1 < we;
-        const int p0 = lane * kItems;
-        const bool full = p0 + kItems <= len;
-        int vv[kItems], ww[kItems];
+        int* mark = s_mark[warp];
 #pragma unroll
-        for (int k = 0; k < kItems; ++k) {
-            vv[k] = nv[k];
-            ww[k] = nw[k];
-        }
-        if (c1 < we) load_chunk(c1, nv, nw);
-
-        // row of every entry: mark row starts inside the chunk, then max-scan
-#pragma unroll
-        for (int i = lane; i < kChunk; i += 32) s_mark[i] = (i == 0) ? r_cur : -1;
+        for (int i = lane; i < kChunk; i += 32) mark[i] = (i == 0) ? r0 : -1;
         __syncwarp();
-        int carry = r_cur;
-        for (long long rb = (long long)r_cur + 1;; rb += 32) {
-            const long long r = rb + lane;
-            bool active = false;
-            if (r < P.n) {
-                const long long s = __ldg(P.nindex + r);
-                if (s < c1) {
-                    active = true;
-                    if (s >= c0) atomicMax(&s_mark[s - c0], (int)r);
-                    else err = 1;   // nindex decreasing
-                } else if (s == c1 && need_carry) {
-                    active = true;
-                }
+        for (int rb = r0 + 1; rb <= r_last; rb += 32) {
+            const int r = rb + lane;
+            if (r <= r_last) {
+                const long long s = P.nindex[r];
+                if (s >= c0 && s < c1) atomicMax(&mark[s - c0], r);
+                else if (s < c0) err = true;
             }
-            const int na = __popc(__ballot_sync(kFull, active));
-            if (na > 0) carry = (int)(rb + na - 1);
-            if (na < 32) break;
         }
         __syncwarp();
         int row[kItems];
 #pragma unroll
-        for (int k = 0; k < kItems; ++k) row[k] = s_mark[p0 + k];
-        __syncwarp();
-        warp_max_scan(row);
+        for (int k = 0; k < kItems; ++k) row[k] = mark[p0 + k];
+        // inclusive max-scan over the warp's 128 positions
+#pragma unroll
+        for (int k = 1; k < kItems; ++k) row[k] = max(row[k], row[k - 1]);
+        int incl = row[kItems - 1];
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int y = __shfl_up_sync(kFull, incl, o);
+            if (lane >= o) incl = max(incl, y);
+        }
+        int excl = __shfl_up_sync(kFull, incl, 1);
+        if (lane == 0) excl = INT_MIN;
+#pragma unroll
+        for (int k = 0; k < kItems; ++k) row[k] = max(row[k], excl);
 
         if (PH == 1) {   // every in_mst byte is written once, here (Alg. 1 "not in MST")
-            if (P.vec_ok && full) {
+            if (p0 + kItems <= len) {
                 __stcs(reinterpret_cast<unsigned*>(P.in_mst + c0 + p0), 0u);
             } else {
 #pragma unroll
@@ -208,36 +301,56 @@ __device__ __forceinline__ void populate(const Params& P, long long wb, long lon
                     if (p0 + k < len) P.in_mst[c0 + p0 + k] = 0;
             }
         }
-
-        int4 t[kItems];
-        bool keep[kItems];
-        int prev_u = -1, prev_p = -1;
+        bool cand[kItems];
+#pragma unroll
+        for (int k = 0; k < kItems; ++k) {
+            const bool valid = p0 + k < len;
+            const bool in_range = (unsigned)vv[k] < (unsigned)P.n;
+            if (valid && !in_range) err = true;
+            const bool canon = valid && in_range && row[k] < vv[k];   // L4: one direction only
+            const bool heavy = filtered && ww[k] >= T;                // L6 threshold condition
+            if (PH == 1) {
+                canon_cnt += canon;
+                heavy_cnt += (canon && heavy);
+                cand[k] = canon && !heavy;
+            } else {
+                cand[k] = canon && heavy;
+            }
+        }
+        int pk[kItems], qk[kItems];
+#pragma unroll
+        for (int k = 0; k < kItems; ++k) {
+            pk[k] = row[k];
+            qk[k] = vv[k];
+        }
+        if (PH == 2) {   // set(v), set(n): one load each after k_flatten
+#pragma unroll
+            for (int k = 0; k < kItems; ++k) {
+                if (cand[k]) {
+                    pk[k] = (k > 0 && cand[k - 1] && row[k] == row[k - 1]) ? -1 : __ldca(P.parent + row[k]);
+                    qk[k] = __ldca(P.parent + vv[k]);
+                }
+            }
+#pragma unroll
+            for (int k = 1; k < kItems; ++k)
+                if (pk[k] == -1) pk[k] = pk[k - 1];
+            if (!P.flatten) {
+#pragma unroll
+                for (int k = 0; k < kItems; ++k) {
+                    if (cand[k]) {
+                        pk[k] = find_root(P.parent, pk[k], P.halving != 0);
+                        qk[k] = find_root(P.parent, qk[k], P.halving != 0);
+                    }
+                }
+            }
+        }
 #pragma unroll
         for (int k = 0; k < kItems; ++k) {
             const long long j = c0 + p0 + k;
-            const bool valid = p0 + k < len;
-            const int u = row[k], v = vv[k], w = ww[k];
-            const bool in_range = (unsigned)v < (unsigned)P.n;
-            if (valid && !in_range) err = 1;
-            const bool canon = valid && in_range && u < v;       // L4: one direction only
-            int p = u, q = v;
-            bool kk = false;
-            if (PH == 1) {
-                const bool heavy = filtered && w >= T;            // L6 threshold condition
-                canon_cnt += canon;
-                heavy_cnt += (canon && heavy);
-                kk = canon && !heavy;
-            } else if (canon && filtered && w >= T) {
-                p = (u == prev_u) ? prev_p : find_root(P.parent, u, halving);   // set(v)
-                prev_u = u;
-                prev_p = p;
-                q = find_root(P.parent, v, halving);                            // set(n)
-                kk = p != q;                                      // filtered out otherwise
-            }
-            t[k] = make_int4(p, q, w, (int)(unsigned)j);
-            keep[k] = kk;
+            t[k] = make_int4(pk[k], qk[k], ww[k], (int)(unsigned)j);
+            keep[k] = cand[k] && pk[k] != qk[k];                  // phase 2: the filter
         }
-        // L20: the lane's entries come in row order, so merge equal p first
+        // L19-21: the lane's entries come in row order, so merge equal p first
         long long best = kInf;
         int bp = -1;
 #pragma unroll
@@ -254,12 +367,76 @@ __device__ __forceinline__ void populate(const Params& P, long long wb, long lon
         }
         if (bp >= 0) record_min(K + bp, best, guard);
 #pragma unroll
-        for (int k = 0; k < kItems; ++k)                          // L21
+        for (int k = 0; k < kItems; ++k)
             if (keep[k]) record_min(K + t[k].y, make_key(t[k].z, (unsigned)t[k].w), guard);
-        warp_emit(t, keep, out, s_out);                          // L7
-        r_cur = carry;
+    }
+    // L7: one arena reservation per warp
+    unsigned m[kItems];
+    int off[kItems];
+    int tot = 0;
+#pragma unroll
+    for (int i = 0; i < kItems; ++i) {
+        m[i] = __ballot_sync(kFull, keep[i]);
+        off[i] = tot;
+        tot += __popc(m[i]);
+    }
+    int base = 0;
+    if (lane == 0 && tot) base = atomicAdd(&P.in->arena_cnt[arena], tot);
+    base = __shfl_sync(kFull, base, 0);
+    const unsigned lt = (1u << lane) - 1u;
+#pragma unroll
+    for (int i = 0; i < kItems; ++i)
+        if (keep[i]) __stcg(out + base + off[i] + __popc(m[i] & lt), t[i]);
+    if (err) atomicExch(&P.st->status, ECL_MST_ERR_INPUT);
+    if (PH == 1) {   // |E| and the deferred count, one atomic pair per CTA
+        canon_cnt = warp_sum(canon_cnt);
+        heavy_cnt = warp_sum(heavy_cnt);
+        if (lane == 0) {
+            s_canon[warp] = canon_cnt;
+            s_heavy[warp] = heavy_cnt;
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            long long cs = 0, hs = 0;
+            for (int w = 0; w < kPopWarps; ++w) {
+                cs += s_canon[w];
+                hs += s_heavy[w];
+            }
+            const int a = (int)(blockIdx.x % P.G);
+            if (cs) atomicAdd(reinterpret_cast<unsigned long long*>(&P.in->arena_canon[a]), (unsigned long long)cs);
+            if (hs) atomicAdd(reinterpret_cast<unsigned long long*>(&P.in->arena_heavy[a]), (unsigned long long)hs);
+        }
     }
 }
+
+// ---------------------------------------------------------------------------
+// k_flatten: parent[v] = find(v) before the phase-2 populate, so the phase-2
+// populate can use parent[x] as set(x) with one load.  Asynchronous pointer
+// jumping in which every slot has exactly one writer (the thread that owns
+// v): path halving is NOT used here, because another thread's halving store
+// could land after the owner's final store and leave v pointing at a
+// non-root ancestor.  Each owner walks its own pointer up; owners of the
+// vertices above it shorten theirs concurrently (reads go through L2 to see
+// that), so the walks shrink geometrically.  Roots never change here.
+// ---------------------------------------------------------------------------
+__global__ void __launch_bounds__(256) k_flatten(Params P) {
+    if (!phase2_needed(P) || !P.flatten) return;
+    const long long stride = (long long)gridDim.x * blockDim.x;
+    int* __restrict__ parent = P.parent;
+    for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < P.n; v += stride) {
+        int p = __ldcg(parent + v);
+        while (true) {
+            const int pp = __ldcg(parent + p);
+            if (pp == p) break;
+            __stcg(parent + v, pp);
+            p = pp;
+        }
+    }
+}
+
+// ---------------------------------------------------------------------------
+// rounds: pass A / pass B over the CTA's arena
+// ---------------------------------------------------------------------------
 
 // L14-23 of one round over the CTA's worklist slice: in[0, cnt) -> out.
 __device__ __forceinline__ void passA(const Params& P, const int4* __restrict__ in, int cnt,
@@ -355,169 +532,83 @@ __device__ __forceinline__ void passB(const Params& P, const int4* __restrict__ 
     }
 }
 
-// per-CTA end of a stage (diagnostics; P.trace is null unless opts.trace)
-__device__ __forceinline__ void trace_cta(const Params& P, int slot) {
-    if (P.trace && slot < kTraceSlots) {
-        __syncthreads();
-        if (threadIdx.x == 0) P.trace[(long long)slot * kMaxGrid + blockIdx.x] = (long long)globaltimer_ns();
-    }
-}
-
-__device__ __forceinline__ void stamp(const Params& P, int slot) {
-    if (blockIdx.x == 0 && threadIdx.x == 0 && slot < 2 * ECL_MST_MAX_ROUNDS + 4)
-        P.st->t_ns[slot] = (long long)globaltimer_ns();
-}
-
-__global__ void __launch_bounds__(kBlock, 2) mst_persistent(Params P) {
+template <int PH>
+__global__ void __launch_bounds__(kBlock, 2) k_rounds(Params P) {
     cg::grid_group grid = cg::this_grid();
-    __shared__ int s_mark[kWarps][kChunk];
     __shared__ int s_out;
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int tid = threadIdx.x, lane = tid & 31;
     const bool b0 = blockIdx.x == 0;
     ecl_mst_stats* st = P.st;
-    const long long t_start = (b0 && tid == 0) ? (long long)globaltimer_ns() : 0;
-    const long long cta_begin = min(P.M, (long long)blockIdx.x * kWarps * P.sub);
-    const long long wb = min(P.M, cta_begin + warp * P.sub);
-    const long long we = min(P.M, wb + P.sub);
-    int err = 0;
-
-    // ---------------- init (Alg. 1) ----------------
-    for (long long v = (long long)blockIdx.x * kBlock + tid; v < P.n; v += (long long)gridDim.x * kBlock) {
-        P.parent[v] = (int)v;
-        P.key[v] = kInf;
+    if (PH == 2 && !phase2_needed(P)) return;
+    int g = (PH == 1) ? 0 : __ldcg(&P.in->g_end) + 1;
+    if (g >= ECL_MST_MAX_ROUNDS) {
+        if (b0 && tid == 0) atomicExch(&st->status, ECL_MST_ERR_INPUT);
+        return;
     }
-    const int r_first = (wb < we) ? warp_row_of(P.nindex, P.n, wb) : 0;
-    if (b0) {
-        long long* words = reinterpret_cast<long long*>(st);
-        for (int i = tid; i < (int)(sizeof(ecl_mst_stats) / 8); i += kBlock) words[i] = 0;
-        __syncthreads();
-        if (warp == 1) {
-            // filter decision (P:143-145, P:152; readings Q5-Q7)
-            const bool filtered = P.filter_mode < 0 ? (P.M >= 4LL * P.n) : (P.filter_mode != 0);
-            int T = INT_MAX;
-            if (filtered) {
-                if (P.threshold_mode == 1) {
-                    T = P.threshold_value;
-                } else {
-                    int w = INT_MAX;
-                    if (lane < 20) {
-                        const unsigned long long h = splitmix64(P.seed * 0x100000001B3ull + (unsigned long long)lane);
-                        w = __ldg(P.eweight + (long long)(h % (unsigned long long)P.M));
-                    }
-                    int rank = 0;
-                    for (int s = 0; s < 20; ++s) {
-                        const int ws = __shfl_sync(kFull, w, s);
-                        if (lane < 20 && (ws < w || (ws == w && s < lane))) ++rank;
-                    }
-                    long long kpos = (80LL * P.n) / P.M;   // c|V| lightest of M entries: 20 * 4n / M
-                    if (kpos > 19) kpos = 19;
-                    const unsigned b = __ballot_sync(kFull, lane < 20 && rank == (int)kpos);
-                    T = __shfl_sync(kFull, w, __ffs(b) - 1);
-                }
-            }
-            if (lane == 0) {
-                st->filtered = filtered ? 1 : 0;
-                st->threshold = T;
-                st->grid = gridDim.x;
-                st->block = kBlock;
-                st->phase2_round = -1;
-                if (P.nindex[0] != 0 || P.nindex[P.n] != P.M) err = 1;
-            }
+    stamp(P, 4 + 2 * g);                      // populate done
+    const int b = blockIdx.x;
+    int4* wl[2] = {P.wl0 + (long long)b * P.cap, P.wl1 + (long long)b * P.cap};
+    if (tid == 0) {
+        // read once, then reset for the phase-2 populate: every thread takes
+        // the count from s_out (a per-thread read could race with the reset)
+        const int c0 = __ldcg(&P.in->arena_cnt[b]);
+        s_out = c0;
+        if (c0) atomicAdd(reinterpret_cast<unsigned long long*>(&st->live[g]), (unsigned long long)c0);
+        if (PH == 1) {
+            const long long cs = __ldcg(&P.in->arena_canon[b]), hs = __ldcg(&P.in->arena_heavy[b]);
+            if (cs) atomicAdd(reinterpret_cast<unsigned long long*>(&st->canonical_edges), (unsigned long long)cs);
+            if (hs) atomicAdd(reinterpret_cast<unsigned long long*>(&st->heavy_edges), (unsigned long long)hs);
         }
-        if (tid == 0) P.in->done = 0u;
+        P.in->arena_cnt[b] = 0;               // ready for the phase-2 populate
+        if (b0 && PH == 2) st->phase2_round = g;
     }
-    trace_cta(P, 1);
+    __syncthreads();
+    int cnt = s_out;
+    trace_cta(P, 4 + 2 * g);
     grid.sync();
-    const bool filtered = __ldcg(&st->filtered) != 0;
-    const int T = __ldcg(&st->threshold);
-    if (b0 && tid == 0) {
-        st->t_ns[0] = t_start;
-        st->t_ns[1] = (long long)globaltimer_ns();
-    }
-
-    long long canon_cnt = 0, heavy_cnt = 0, wsum = 0, wcnt = 0;
-    int4* wl[2] = {P.wl0 + cta_begin, P.wl1 + cta_begin};
-    int cur = 0, g = 0, cnt = 0;
+    long long wsum = 0, wcnt = 0;
+    int cur = 0;
     bool overflow = false;
-    for (int ph = 1; ph <= 2 && !overflow; ++ph) {
-        if (ph == 2) {
-            if (!filtered || __ldcg(&st->heavy_edges) == 0) break;
-            if (g + 1 >= ECL_MST_MAX_ROUNDS) { overflow = true; break; }
-            if (P.flatten) {   // compress every path once: phase-2 finds become one hop
-                for (long long v = (long long)blockIdx.x * kBlock + tid; v < P.n; v += (long long)gridDim.x * kBlock) {
-                    const int r = find_root(P.parent, (int)v, true);
-                    if (r != (int)v) P.parent[v] = r;
-                }
-                trace_cta(P, 3);
-                grid.sync();
-                stamp(P, 3);
-            }
-            ++g;
-            if (b0 && tid == 0) st->phase2_round = g;
-        }
+    long long L = __ldcg(&st->live[g]);
+    while (L > 0) {
+        const long long w0 = wcnt;
+        passB(P, wl[cur], cnt, wsum, wcnt);
+        const long long d = warp_sum(wcnt - w0);
+        if (lane == 0 && d) atomicAdd(reinterpret_cast<unsigned long long*>(&st->winners[g]), (unsigned long long)d);
         if (tid == 0) s_out = 0;
-        __syncthreads();
-        if (ph == 1)
-            populate<1>(P, wb, we, r_first, filtered, T, s_mark[warp], wl[cur], &s_out, canon_cnt, heavy_cnt, err);
-        else
-            populate<2>(P, wb, we, r_first, filtered, T, s_mark[warp], wl[cur], &s_out, canon_cnt, heavy_cnt, err);
+        trace_cta(P, 5 + 2 * g);
+        grid.sync();
+        stamp(P, 5 + 2 * g);
+        if (g + 1 >= ECL_MST_MAX_ROUNDS) { overflow = true; break; }
+        ++g;
+        passA(P, wl[cur], cnt, wl[cur ^ 1], &s_out);
+        cur ^= 1;
         __syncthreads();
         cnt = s_out;
         if (tid == 0 && cnt) atomicAdd(reinterpret_cast<unsigned long long*>(&st->live[g]), (unsigned long long)cnt);
-        if (ph == 1) {
-            const long long c = warp_sum(canon_cnt), h = warp_sum(heavy_cnt);
-            if (lane == 0 && c) atomicAdd(reinterpret_cast<unsigned long long*>(&st->canonical_edges), (unsigned long long)c);
-            if (lane == 0 && h) atomicAdd(reinterpret_cast<unsigned long long*>(&st->heavy_edges), (unsigned long long)h);
-        }
         trace_cta(P, 4 + 2 * g);
         grid.sync();
         stamp(P, 4 + 2 * g);
-        long long L = __ldcg(&st->live[g]);
-        while (L > 0) {
-            const long long w0 = wcnt;
-            passB(P, wl[cur], cnt, wsum, wcnt);
-            const long long d = warp_sum(wcnt - w0);
-            if (lane == 0 && d) atomicAdd(reinterpret_cast<unsigned long long*>(&st->winners[g]), (unsigned long long)d);
-            if (tid == 0) s_out = 0;
-            trace_cta(P, 5 + 2 * g);
-            grid.sync();
-            stamp(P, 5 + 2 * g);
-            if (g + 1 >= ECL_MST_MAX_ROUNDS) { overflow = true; break; }
-            ++g;
-            passA(P, wl[cur], cnt, wl[cur ^ 1], &s_out);
-            cur ^= 1;
-            __syncthreads();
-            cnt = s_out;
-            if (tid == 0 && cnt) atomicAdd(reinterpret_cast<unsigned long long*>(&st->live[g]), (unsigned long long)cnt);
-            trace_cta(P, 4 + 2 * g);
-            grid.sync();
-            stamp(P, 4 + 2 * g);
-            L = __ldcg(&st->live[g]);
-        }
+        L = __ldcg(&st->live[g]);
     }
-    if (overflow) err = 1;
-
-    // ---------------- finalise ----------------
     const long long s = warp_sum(wsum), c = warp_sum(wcnt);
     if (lane == 0) {
         if (s) atomicAdd(reinterpret_cast<unsigned long long*>(&st->total_weight), (unsigned long long)s);
         if (c) atomicAdd(reinterpret_cast<unsigned long long*>(&st->msf_edges), (unsigned long long)c);
     }
-    if (err) atomicExch(&st->status, ECL_MST_ERR_INPUT);
-    __threadfence();
-    __syncthreads();
-    if (tid == 0) {
-        if (b0) {
-            st->rounds = g + 1;
-            st->t_ns[2] = (long long)globaltimer_ns();
-        }
-        const unsigned ticket = atomicAdd(&P.in->done, 1u);
-        if (ticket == gridDim.x - 1) {
-            __threadfence();
-            const long long tot = *reinterpret_cast<volatile long long*>(&st->total_weight);
-            const int status = *reinterpret_cast<volatile int*>(&st->status);
-            *P.total_out = status ? LLONG_MIN : tot;
-        }
+    if (b0 && tid == 0) {
+        P.in->g_end = g;
+        st->rounds = g + 1;
+        if (overflow) atomicExch(&st->status, ECL_MST_ERR_INPUT);
+    }
+}
+
+__global__ void k_finalize(Params P) {
+    if (threadIdx.x == 0) {
+        ecl_mst_stats* st = P.st;
+        st->t_ns[2] = (long long)globaltimer_ns();
+        const int status = *reinterpret_cast<volatile int*>(&st->status);
+        *P.total_out = status ? LLONG_MIN : *reinterpret_cast<volatile long long*>(&st->total_weight);
     }
 }
 
@@ -556,7 +647,7 @@ static int device_info(DevInfo* out) {
         int sms = 0, coop = 0, occ = 0;
         e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
         if (e == cudaSuccess) e = cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, dev);
-        if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, mst_persistent, kBlock, 0);
+        if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_rounds<1>, kBlock, 0);
         if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "device query: %s", cudaGetErrorString(e));
         if (!coop || occ < 1) return fail(ECL_MST_ERR_CUDA, "cooperative launch unsupported (coop=%d occ=%d)", coop, occ);
         g_dev[dev].sms = sms;
@@ -583,7 +674,7 @@ void ecl_mst_default_options(ecl_mst_options* o) {
     o->threshold_mode = 0;
     o->threshold = 0;
     o->path_halving = 1;
-    o->atomic_guards = 1;
+    o->atomic_guards = -1;
     o->flatten = 1;
     o->max_ctas = 0;
     o->trace = 0;
@@ -623,27 +714,22 @@ int ecl_mst_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t* n
     DevInfo di;
     int rc = device_info(&di);
     if (rc) return rc;
-    const long long max_g = (long long)di.sms * di.occ;
-    long long G = max_g;
-    const long long chunks = (M + kChunk - 1) / kChunk;
-    if (G * kWarps > chunks) G = (chunks + kWarps - 1) / kWarps;   // small graphs: fewer CTAs
+    const long long nchunks = ceil_div(M, kChunk);
+    long long G = (long long)di.sms * di.occ;
     if (o.max_ctas > 0 && G > o.max_ctas) G = o.max_ctas;
+    if (G > nchunks) G = nchunks;                 // small graphs: fewer, fuller arenas
     if (G > kMaxGrid) G = kMaxGrid;
     if (G < 1) G = 1;
-    long long sub = (M + G * kWarps - 1) / (G * kWarps);
-    sub = (sub + kItems - 1) / kItems * kItems;
-    // per-CTA worklist counts are int: keep a CTA's slice below 2^30 entries
-    while (sub * kWarps >= (1LL << 30)) {
-        if (G >= max_g) return fail(ECL_MST_ERR_TOO_LARGE, "graph needs more CTAs than fit");
-        ++G;
-        sub = (M + G * kWarps - 1) / (G * kWarps);
-        sub = (sub + kItems - 1) / kItems * kItems;
-    }
+    const long long cap = ceil_div(nchunks, G) * kChunk;
+    if (cap >= (1LL << 30)) return fail(ECL_MST_ERR_TOO_LARGE, "arena of %lld tuples too large", cap);
+    if (G * cap > L.wl_cap) return fail(ECL_MST_ERR_WORKSPACE, "internal: arenas exceed worklist capacity");
 
     Params P;
     P.n = n;
     P.M = M;
-    P.sub = sub;
+    P.nchunks = nchunks;
+    P.G = (int)G;
+    P.cap = cap;
     P.nindex = reinterpret_cast<const long long*>(nindex);
     P.nlist = nlist;
     P.eweight = eweight;
@@ -652,6 +738,7 @@ int ecl_mst_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t* n
     P.st = reinterpret_cast<ecl_mst_stats*>(ws + L.stats);
     P.in = reinterpret_cast<Internal*>(ws + L.internal);
     P.trace = o.trace ? reinterpret_cast<long long*>(ws + L.trace) : nullptr;
+    P.rowstart = reinterpret_cast<int*>(ws + L.rowstart);
     P.key = reinterpret_cast<long long*>(ws + L.key);
     P.parent = reinterpret_cast<int*>(ws + L.parent);
     P.wl0 = reinterpret_cast<int4*>(ws + L.wl0);
@@ -661,14 +748,36 @@ int ecl_mst_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t* n
     P.threshold_mode = o.threshold_mode;
     P.threshold_value = o.threshold;
     P.halving = o.path_halving ? 1 : 0;
-    P.guards = o.atomic_guards ? 1 : 0;
+    P.guards = o.atomic_guards < 0 ? -1 : (o.atomic_guards ? 1 : 0);
     P.flatten = o.flatten ? 1 : 0;
-    P.vec_ok = (reinterpret_cast<uintptr_t>(nlist) % 16 == 0) && (reinterpret_cast<uintptr_t>(eweight) % 16 == 0) &&
-               (reinterpret_cast<uintptr_t>(in_mst_out) % 4 == 0);
+    if ((reinterpret_cast<uintptr_t>(nlist) | reinterpret_cast<uintptr_t>(eweight)) % 16 ||
+        reinterpret_cast<uintptr_t>(in_mst_out) % 4)
+        return fail(ECL_MST_ERR_INVALID, "nlist/eweight must be 16-byte and in_mst 4-byte aligned");
+
+    const long long init_blocks = std::min<long long>(ceil_div((long long)n, 256), (long long)di.sms * 8);
+    const long long pop_blocks = ceil_div(nchunks, kPopWarps);
+    if (pop_blocks > INT_MAX) return fail(ECL_MST_ERR_TOO_LARGE, "too many populate CTAs");
     void* args[] = {&P};
-    cudaError_t e = cudaLaunchCooperativeKernel(reinterpret_cast<const void*>(mst_persistent), dim3((unsigned)G),
-                                                dim3(kBlock), args, 0, s);
-    if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "cooperative launch (grid %lld): %s", G, cudaGetErrorString(e));
+    cudaError_t e = cudaMemsetAsync(P.st, 0, sizeof(ecl_mst_stats), s);
+    if (e == cudaSuccess) {
+        k_init<<<(unsigned)std::max<long long>(init_blocks, 1), 256, 0, s>>>(P);
+        k_populate<1><<<(unsigned)pop_blocks, kPopBlock, 0, s>>>(P);
+        e = cudaGetLastError();
+    }
+    if (e == cudaSuccess)
+        e = cudaLaunchCooperativeKernel(reinterpret_cast<const void*>(k_rounds<1>), dim3((unsigned)G), dim3(kBlock), args, 0, s);
+    if (e == cudaSuccess) {
+        k_flatten<<<(unsigned)std::max<long long>(init_blocks, 1), 256, 0, s>>>(P);
+        k_populate<2><<<(unsigned)pop_blocks, kPopBlock, 0, s>>>(P);
+        e = cudaGetLastError();
+    }
+    if (e == cudaSuccess)
+        e = cudaLaunchCooperativeKernel(reinterpret_cast<const void*>(k_rounds<2>), dim3((unsigned)G), dim3(kBlock), args, 0, s);
+    if (e == cudaSuccess) {
+        k_finalize<<<1, 32, 0, s>>>(P);
+        e = cudaGetLastError();
+    }
+    if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "launch (G=%lld): %s", G, cudaGetErrorString(e));
     return ECL_MST_OK;
 }
 

@@ -48,7 +48,7 @@ def test_workspace_bytes(lib):
 
 def test_argument_validation_without_gpu(lib):
     o = _native.default_options()
-    assert o.filter == -1 and o.path_halving == 1 and o.atomic_guards == 1 and o.flatten == 1
+    assert o.filter == -1 and o.path_halving == 1 and o.atomic_guards == -1 and o.flatten == 1
     assert o.seed == 0x5EED
     rc = lib.ecl_mst_device(-1, 0, None, None, None, None, None, None, 0, None, None)
     assert rc == _native.ERR_INVALID
