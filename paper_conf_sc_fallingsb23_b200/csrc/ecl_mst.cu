@@ -52,6 +52,8 @@ namespace eclmst {
 constexpr int kMaxGrid = 4096;                 // CTAs of k_rounds (= arenas), upper bound
 constexpr int kPopWarps = 8;                   // warps per k_populate CTA (one chunk each)
 constexpr int kPopBlock = 32 * kPopWarps;
+constexpr int kMaxPopWarps = 65536;            // populate warps (= worklist regions), upper bound
+constexpr int kMaxRegionsPerCta = 256;         // regions a k_rounds CTA starts from
 constexpr int kTraceSlots = 2 * ECL_MST_MAX_ROUNDS + 4;
 static_assert(kMaxGrid == ECL_MST_TRACE_CTAS, "trace layout");
 
@@ -60,13 +62,10 @@ struct Internal {
     int g_cur;                         // first global round of the running phase
     int g_end;                         // last global round of the finished phase
     int pad0;
-    int arena_cnt[kMaxGrid];           // tuples emitted into each arena by k_populate
-    long long arena_canon[kMaxGrid];   // canonical edges seen, per arena (phase 1)
-    long long arena_heavy[kMaxGrid];   // heavy canonical edges, per arena (phase 1)
 };
 
 struct Layout {
-    size_t stats, internal, trace, rowstart, key, parent, wl0, wl1, total;
+    size_t stats, internal, trace, rowstart, region, key, parent, wl0, wl1, total;
     long long wl_cap;                  // tuples per worklist buffer
 };
 
@@ -74,12 +73,12 @@ static inline size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; 
 
 static inline long long ceil_div(long long a, long long b) { return (a + b - 1) / b; }
 
-// worklist tuples needed for G arenas of ceil(nchunks/G)*kChunk tuples, for
-// any G <= min(kMaxGrid, nchunks)
+// worklist tuples needed for W populate regions of ceil(nchunks/W)*kChunk
+// tuples, for any W <= min(kMaxPopWarps, nchunks)
 static inline long long wl_capacity(long long M) {
     const long long nchunks = ceil_div(M, kChunk);
-    const long long gmax = nchunks < kMaxGrid ? nchunks : kMaxGrid;
-    return (nchunks + gmax) * (long long)kChunk;
+    const long long wmax = nchunks < kMaxPopWarps ? nchunks : kMaxPopWarps;
+    return (nchunks + wmax) * (long long)kChunk;
 }
 
 static inline Layout layout_for(int64_t n, int64_t M) {
@@ -91,6 +90,7 @@ static inline Layout layout_for(int64_t n, int64_t M) {
     L.internal = off; off = align_up(off + sizeof(Internal), 256);
     L.trace = off;    off = align_up(off + sizeof(long long) * kTraceSlots * kMaxGrid, 256);
     L.rowstart = off; off = align_up(off + sizeof(int) * (size_t)(nchunks + 1), 256);
+    L.region = off;   off = align_up(off + sizeof(int4) * (size_t)kMaxPopWarps, 256);
     L.key = off;      off = align_up(off + sizeof(long long) * (size_t)n, 256);
     L.parent = off;   off = align_up(off + sizeof(int) * (size_t)n, 256);
     L.wl0 = off;      off = align_up(off + sizeof(int4) * (size_t)L.wl_cap, 256);
@@ -104,7 +104,9 @@ struct Params {
     long long M;
     long long nchunks;                // ceil(M / kChunk)
     int G;                            // k_rounds CTAs = arenas
-    long long cap;                    // tuples per arena
+    long long cap;                    // tuples per arena (k_rounds worklists)
+    int W;                            // populate warps = regions of wl0
+    long long rcap;                   // tuples per region
     const long long* __restrict__ nindex;
     const int* __restrict__ nlist;
     const int* __restrict__ eweight;
@@ -114,6 +116,7 @@ struct Params {
     Internal* in;
     long long* trace;                 // [kTraceSlots][kMaxGrid] or null
     int* rowstart;                    // row of CSR entry c*kChunk, per chunk
+    int4* region;                     // per populate warp: {tuples, canonical, heavy, 0}
     long long* key;
     int* parent;
     int4* wl0;
@@ -141,8 +144,10 @@ __device__ __forceinline__ void trace_cta(const Params& P, int slot) {
 }
 
 // phase 2 runs iff filtering is on and phase 1 deferred at least one edge
+// (read-only within the kernels that ask: one L1 line per SM, not one L2
+// slice hammered by every warp of the grid)
 __device__ __forceinline__ bool phase2_needed(const Params& P) {
-    return __ldcg(&P.st->filtered) != 0 && __ldcg(&P.st->heavy_edges) != 0;
+    return __ldg(&P.st->filtered) != 0 && __ldg(&P.st->heavy_edges) != 0;
 }
 
 // ---------------------------------------------------------------------------
@@ -163,12 +168,6 @@ __global__ void __launch_bounds__(256) k_init(Params P) {
     }
     if (blockIdx.x == 0) {
         ecl_mst_stats* st = P.st;   // zeroed by a memset node just before this kernel
-        for (int i = tid; i < P.G; i += blockDim.x) {
-            P.in->arena_cnt[i] = 0;
-            P.in->arena_canon[i] = 0;
-            P.in->arena_heavy[i] = 0;
-        }
-        __syncthreads();
         if (warp == 0) {
             // filter decision (readings Q5-Q7)
             const bool filtered = P.filter_mode < 0 ? (P.M >= 4LL * P.n) : (P.filter_mode != 0);
@@ -216,38 +215,39 @@ __global__ void __launch_bounds__(256) k_init(Params P) {
 template <int PH>
 __global__ void __launch_bounds__(kPopBlock, 8) k_populate(Params P) {
     __shared__ int s_mark[kPopWarps][kChunk];
-    __shared__ long long s_canon[kPopWarps], s_heavy[kPopWarps];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     if (PH == 2 && !phase2_needed(P)) return;
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         if (PH == 1) P.st->t_ns[1] = (long long)globaltimer_ns();   // init done
         else P.st->t_ns[3] = (long long)globaltimer_ns();           // flatten done
     }
-    const bool filtered = __ldcg(&P.st->filtered) != 0;
-    const int T = __ldcg(&P.st->threshold);
+    const bool filtered = __ldg(&P.st->filtered) != 0;
+    const int T = __ldg(&P.st->threshold);
     const bool guard = (P.guards > 0) || (P.guards < 0 && PH == 2);
     long long* __restrict__ K = P.key;
-    const long long c = (long long)blockIdx.x * kPopWarps + warp;
-    // chunk-level round robin over the arenas: every arena samples the whole
-    // CSR, so the round kernel's CTAs start with balanced work even where
-    // the density of u < v entries drifts along the rows
-    const int arena = (int)(c % P.G);
-    int4* out = P.wl0 + (long long)arena * P.cap;
+    int* __restrict__ parent = P.parent;
+    // warp w takes chunks w, w + W, ... (an even sample of the whole CSR, so
+    // every region -- and every k_rounds CTA -- gets the same mix even where
+    // the density of u < v entries drifts along the rows) and appends its
+    // tuples densely to its own region: no atomics, no CTA barrier.
+    const int w = blockIdx.x * kPopWarps + warp;
+    if (w >= P.W) return;
+    int4* const out = P.wl0 + (long long)w * P.rcap;
+    int cnt = 0, canon_cnt = 0, heavy_cnt = 0;
+    bool err = false;
+    for (long long c = w; c < P.nchunks; c += P.W) {
     bool keep[kItems];
     int4 t[kItems];
-    long long canon_cnt = 0, heavy_cnt = 0;
-    bool err = false;
 #pragma unroll
     for (int k = 0; k < kItems; ++k) keep[k] = false;
-
     if (c < P.nchunks) {
         const long long c0 = c * kChunk;
         const long long c1 = min(c0 + (long long)kChunk, P.M);
         const int len = (int)(c1 - c0);
         const int p0 = lane * kItems;
         // rows of this chunk: r0 = row of entry c0; rows r0+1 .. r_last start inside
-        const int r0 = P.rowstart[c];
-        const int r_last = (c + 1 < P.nchunks) ? P.rowstart[c + 1] : P.n - 1;
+        const int r0 = __ldg(P.rowstart + c);
+        const int r_last = (c + 1 < P.nchunks) ? __ldg(P.rowstart + c + 1) : P.n - 1;
         int vv[kItems], ww[kItems];
         if (p0 + kItems <= len) {
             const int4 a = __ldcs(reinterpret_cast<const int4*>(P.nlist + c0 + p0));
@@ -327,8 +327,8 @@ __global__ void __launch_bounds__(kPopBlock, 8) k_populate(Params P) {
 #pragma unroll
             for (int k = 0; k < kItems; ++k) {
                 if (cand[k]) {
-                    pk[k] = (k > 0 && cand[k - 1] && row[k] == row[k - 1]) ? -1 : __ldca(P.parent + row[k]);
-                    qk[k] = __ldca(P.parent + vv[k]);
+                    pk[k] = (k > 0 && cand[k - 1] && row[k] == row[k - 1]) ? -1 : __ldca(parent + row[k]);
+                    qk[k] = __ldca(parent + vv[k]);
                 }
             }
 #pragma unroll
@@ -338,8 +338,8 @@ __global__ void __launch_bounds__(kPopBlock, 8) k_populate(Params P) {
 #pragma unroll
                 for (int k = 0; k < kItems; ++k) {
                     if (cand[k]) {
-                        pk[k] = find_root(P.parent, pk[k], P.halving != 0);
-                        qk[k] = find_root(P.parent, qk[k], P.halving != 0);
+                        pk[k] = find_root(parent, pk[k], P.halving != 0);
+                        qk[k] = find_root(parent, qk[k], P.halving != 0);
                     }
                 }
             }
@@ -370,7 +370,7 @@ __global__ void __launch_bounds__(kPopBlock, 8) k_populate(Params P) {
         for (int k = 0; k < kItems; ++k)
             if (keep[k]) record_min(K + t[k].y, make_key(t[k].z, (unsigned)t[k].w), guard);
     }
-    // L7: one arena reservation per warp
+    // L7: append the chunk's tuples to the warp's region
     unsigned m[kItems];
     int off[kItems];
     int tot = 0;
@@ -380,56 +380,50 @@ __global__ void __launch_bounds__(kPopBlock, 8) k_populate(Params P) {
         off[i] = tot;
         tot += __popc(m[i]);
     }
-    int base = 0;
-    if (lane == 0 && tot) base = atomicAdd(&P.in->arena_cnt[arena], tot);
-    base = __shfl_sync(kFull, base, 0);
     const unsigned lt = (1u << lane) - 1u;
 #pragma unroll
     for (int i = 0; i < kItems; ++i)
-        if (keep[i]) __stcg(out + base + off[i] + __popc(m[i] & lt), t[i]);
+        if (keep[i]) __stcg(out + cnt + off[i] + __popc(m[i] & lt), t[i]);
+    cnt += tot;
+    }
     if (err) atomicExch(&P.st->status, ECL_MST_ERR_INPUT);
-    if (PH == 1) {   // |E| and the deferred count, one atomic pair per CTA
+    if (PH == 1) {   // |E| and the deferred count of this warp's chunks
         canon_cnt = warp_sum(canon_cnt);
         heavy_cnt = warp_sum(heavy_cnt);
-        if (lane == 0) {
-            s_canon[warp] = canon_cnt;
-            s_heavy[warp] = heavy_cnt;
-        }
-        __syncthreads();
-        if (threadIdx.x == 0) {
-            long long cs = 0, hs = 0;
-            for (int w = 0; w < kPopWarps; ++w) {
-                cs += s_canon[w];
-                hs += s_heavy[w];
-            }
-            const int a = (int)(blockIdx.x % P.G);
-            if (cs) atomicAdd(reinterpret_cast<unsigned long long*>(&P.in->arena_canon[a]), (unsigned long long)cs);
-            if (hs) atomicAdd(reinterpret_cast<unsigned long long*>(&P.in->arena_heavy[a]), (unsigned long long)hs);
-        }
     }
+    if (lane == 0) P.region[w] = make_int4(cnt, canon_cnt, heavy_cnt, 0);
 }
 
 // ---------------------------------------------------------------------------
 // k_flatten: parent[v] = find(v) before the phase-2 populate, so the phase-2
-// populate can use parent[x] as set(x) with one load.  Asynchronous pointer
-// jumping in which every slot has exactly one writer (the thread that owns
-// v): path halving is NOT used here, because another thread's halving store
-// could land after the owner's final store and leave v pointing at a
-// non-root ancestor.  Each owner walks its own pointer up; owners of the
-// vertices above it shorten theirs concurrently (reads go through L2 to see
-// that), so the walks shrink geometrically.  Roots never change here.
+// populate can use parent[x] as set(x) with one load.  Two launches: stage 1
+// compresses with path halving from every vertex (fast, but a halving store
+// of one thread can land after another thread's final root store and leave
+// a vertex one or two hops from its root); stage 2 finishes exactly with
+// owner-only pointer jumping (each slot written by the thread that owns it,
+// reads through L2 to see the others' progress), cheap on the short paths
+// stage 1 leaves.  Roots never change here.
 // ---------------------------------------------------------------------------
+template <int STAGE>
 __global__ void __launch_bounds__(256) k_flatten(Params P) {
     if (!phase2_needed(P) || !P.flatten) return;
     const long long stride = (long long)gridDim.x * blockDim.x;
     int* __restrict__ parent = P.parent;
     for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < P.n; v += stride) {
-        int p = __ldcg(parent + v);
-        while (true) {
-            const int pp = __ldcg(parent + p);
-            if (pp == p) break;
-            __stcg(parent + v, pp);
-            p = pp;
+        if (STAGE == 1) {
+            // fast, racy compression: path halving by everybody (ends close
+            // to, but not always exactly at, one hop)
+            const int r = find_root(parent, (int)v, true);
+            if (r != (int)v) parent[v] = r;
+        } else {
+            // exact: owner-only pointer jumping over the now-short paths
+            int p = __ldcg(parent + v);
+            while (true) {
+                const int pp = __ldcg(parent + p);
+                if (pp == p) break;
+                __stcg(parent + v, pp);
+                p = pp;
+            }
         }
     }
 }
@@ -438,20 +432,69 @@ __global__ void __launch_bounds__(256) k_flatten(Params P) {
 // rounds: pass A / pass B over the CTA's arena
 // ---------------------------------------------------------------------------
 
-// L14-23 of one round over the CTA's worklist slice: in[0, cnt) -> out.
-__device__ __forceinline__ void passA(const Params& P, const int4* __restrict__ in, int cnt,
-                                      int4* __restrict__ out, int* s_out) {
+// A CTA's worklist as a sequence of 128-tuple chunks.  Right after populate
+// it is the CTA's share of the populate regions (regions b, b+G, ..., each a
+// dense run of region[w].x tuples; chunk j maps to a region by a binary
+// search over s_pre); after a pass A it is one compact run of cnt tuples.
+struct Src {
+    const int4* base;   // compact mode
+    int cnt;
+    int nloc;           // number of chunks
+    const int* s_pre;   // region mode (shared memory): chunk prefix per region, or null
+    const int* s_rcnt;  //   tuples per region
+    int nreg;
+    const int4* wl0;
+    long long rcap;
+    int first_w;
+    int G;
+    __device__ __forceinline__ const int4* get(int j, int& count) const {
+        if (!s_pre) {
+            count = min(kChunk, cnt - j * kChunk);
+            return base + (long long)j * kChunk;
+        }
+        int lo = 0, hi = nreg;
+        while (hi - lo > 1) {
+            const int mid = (lo + hi) >> 1;
+            if (s_pre[mid] <= j) lo = mid;
+            else hi = mid;
+        }
+        const int off = j - s_pre[lo];
+        count = min(kChunk, s_rcnt[lo] - off * kChunk);
+        return wl0 + (long long)(first_w + lo * G) * rcap + (long long)off * kChunk;
+    }
+};
+
+__device__ __forceinline__ Src compact_src(const int4* base, int cnt) {
+    Src S;
+    S.base = base;
+    S.cnt = cnt;
+    S.nloc = (cnt + kChunk - 1) / kChunk;
+    S.s_pre = nullptr;
+    S.s_rcnt = nullptr;
+    S.nreg = 0;
+    S.wl0 = nullptr;
+    S.rcap = 0;
+    S.first_w = 0;
+    S.G = 0;
+    return S;
+}
+
+// L14-23 of one round over the CTA's worklist: S -> out (compact).
+__device__ __forceinline__ void passA(const Params& P, const Src& S, int4* __restrict__ out, int* s_out,
+                                      bool guard) {
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const bool halving = P.halving != 0, guard = P.guards != 0;
+    const bool halving = P.halving != 0;
     int* __restrict__ parent = P.parent;
     long long* __restrict__ K = P.key;
-    for (int c = warp * kChunk; c < cnt; c += kWarps * kChunk) {
+    for (int k = warp; k < S.nloc; k += kWarps) {
+        int count;
+        const int4* __restrict__ in = S.get(k, count);
         int4 t[kItems];
         bool keep[kItems];
 #pragma unroll
         for (int i = 0; i < kItems; ++i) {
-            const int idx = c + i * 32 + lane;
-            keep[i] = idx < cnt;
+            const int idx = i * 32 + lane;
+            keep[i] = idx < count;
             t[i] = keep[i] ? __ldcs(in + idx) : make_int4(0, 0, 0, 0);
         }
         int px[kItems], qx[kItems];
@@ -484,20 +527,21 @@ __device__ __forceinline__ void passA(const Params& P, const int4* __restrict__ 
     }
 }
 
-// L27-31 (+ L34-37): check, join, mark over the CTA's worklist slice.
-__device__ __forceinline__ void passB(const Params& P, const int4* __restrict__ wl, int cnt,
-                                      long long& wsum, long long& wcnt) {
+// L27-31 (+ L34-37): check, join, mark over the CTA's worklist.
+__device__ __forceinline__ void passB(const Params& P, const Src& S, long long& wsum, long long& wcnt) {
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     int* __restrict__ parent = P.parent;
     long long* __restrict__ K = P.key;
-    for (int c = warp * kChunk; c < cnt; c += kWarps * kChunk) {
+    for (int k = warp; k < S.nloc; k += kWarps) {
+        int count;
+        const int4* __restrict__ in = S.get(k, count);
         int4 t[kItems];
         bool ok[kItems];
 #pragma unroll
         for (int i = 0; i < kItems; ++i) {
-            const int idx = c + i * 32 + lane;
-            ok[i] = idx < cnt;
-            t[i] = ok[i] ? __ldcg(wl + idx) : make_int4(0, 0, 0, 0);
+            const int idx = i * 32 + lane;
+            ok[i] = idx < count;
+            t[i] = ok[i] ? __ldcg(in + idx) : make_int4(0, 0, 0, 0);
         }
         // Only the id half of each slot is compared: ids are unique per
         // edge, so id equality is key equality (and inf's id half, 2^32-1,
@@ -532,11 +576,23 @@ __device__ __forceinline__ void passB(const Params& P, const int4* __restrict__ 
     }
 }
 
+// guard policy for pass A: "auto" guards only when edges crowd onto
+// few sets.  Each set with a live edge produced exactly one winner last round
+// (mutual pairs: one for two sets), so live / winners estimates the number of
+// edges per set that will atomicMin the same slot.
+__device__ __forceinline__ bool use_guard(const Params& P, long long live, long long winners) {
+    if (P.guards >= 0) return P.guards != 0;
+    return live > 4 * winners;
+}
+
 template <int PH>
 __global__ void __launch_bounds__(kBlock, 2) k_rounds(Params P) {
     cg::grid_group grid = cg::this_grid();
     __shared__ int s_out;
-    const int tid = threadIdx.x, lane = tid & 31;
+    __shared__ long long s_red[3][kWarps];
+    __shared__ int s_pre[kMaxRegionsPerCta + 1];
+    __shared__ int s_rcnt[kMaxRegionsPerCta];
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const bool b0 = blockIdx.x == 0;
     ecl_mst_stats* st = P.st;
     if (PH == 2 && !phase2_needed(P)) return;
@@ -548,22 +604,56 @@ __global__ void __launch_bounds__(kBlock, 2) k_rounds(Params P) {
     stamp(P, 4 + 2 * g);                      // populate done
     const int b = blockIdx.x;
     int4* wl[2] = {P.wl0 + (long long)b * P.cap, P.wl1 + (long long)b * P.cap};
-    if (tid == 0) {
-        // read once, then reset for the phase-2 populate: every thread takes
-        // the count from s_out (a per-thread read could race with the reset)
-        const int c0 = __ldcg(&P.in->arena_cnt[b]);
-        s_out = c0;
-        if (c0) atomicAdd(reinterpret_cast<unsigned long long*>(&st->live[g]), (unsigned long long)c0);
-        if (PH == 1) {
-            const long long cs = __ldcg(&P.in->arena_canon[b]), hs = __ldcg(&P.in->arena_heavy[b]);
-            if (cs) atomicAdd(reinterpret_cast<unsigned long long*>(&st->canonical_edges), (unsigned long long)cs);
-            if (hs) atomicAdd(reinterpret_cast<unsigned long long*>(&st->heavy_edges), (unsigned long long)hs);
+    // the populate output of this CTA: regions w = b, b + G, ... (region mode)
+    Src S;
+    S.base = nullptr;
+    S.cnt = 0;
+    S.s_pre = s_pre;
+    S.s_rcnt = s_rcnt;
+    S.nreg = b < P.W ? (P.W - b + P.G - 1) / P.G : 0;
+    S.wl0 = P.wl0;
+    S.rcap = P.rcap;
+    S.first_w = b;
+    S.G = P.G;
+    {
+        long long canon = 0, heavy = 0;
+        for (int k = tid; k < S.nreg; k += kBlock) {
+            const int4 r = P.region[b + k * P.G];
+            s_rcnt[k] = r.x;
+            canon += r.y;
+            heavy += r.z;
         }
-        P.in->arena_cnt[b] = 0;               // ready for the phase-2 populate
-        if (b0 && PH == 2) st->phase2_round = g;
+        canon = warp_sum(canon);
+        heavy = warp_sum(heavy);
+        if (lane == 0) {
+            s_red[1][warp] = canon;
+            s_red[2][warp] = heavy;
+        }
+        __syncthreads();
+        if (tid == 0) {
+            long long kept = 0;
+            int pre = 0;
+            for (int k = 0; k < S.nreg; ++k) {
+                s_pre[k] = pre;
+                pre += (s_rcnt[k] + kChunk - 1) / kChunk;
+                kept += s_rcnt[k];
+            }
+            s_pre[S.nreg] = pre;
+            canon = heavy = 0;
+            for (int w2 = 0; w2 < kWarps; ++w2) {
+                canon += s_red[1][w2];
+                heavy += s_red[2][w2];
+            }
+            if (kept) atomicAdd(reinterpret_cast<unsigned long long*>(&st->live[g]), (unsigned long long)kept);
+            if (PH == 1) {
+                if (canon) atomicAdd(reinterpret_cast<unsigned long long*>(&st->canonical_edges), (unsigned long long)canon);
+                if (heavy) atomicAdd(reinterpret_cast<unsigned long long*>(&st->heavy_edges), (unsigned long long)heavy);
+            }
+            if (b0 && PH == 2) st->phase2_round = g;
+        }
+        __syncthreads();
+        S.nloc = s_pre[S.nreg];
     }
-    __syncthreads();
-    int cnt = s_out;
     trace_cta(P, 4 + 2 * g);
     grid.sync();
     long long wsum = 0, wcnt = 0;
@@ -572,7 +662,7 @@ __global__ void __launch_bounds__(kBlock, 2) k_rounds(Params P) {
     long long L = __ldcg(&st->live[g]);
     while (L > 0) {
         const long long w0 = wcnt;
-        passB(P, wl[cur], cnt, wsum, wcnt);
+        passB(P, S, wsum, wcnt);
         const long long d = warp_sum(wcnt - w0);
         if (lane == 0 && d) atomicAdd(reinterpret_cast<unsigned long long*>(&st->winners[g]), (unsigned long long)d);
         if (tid == 0) s_out = 0;
@@ -580,12 +670,13 @@ __global__ void __launch_bounds__(kBlock, 2) k_rounds(Params P) {
         grid.sync();
         stamp(P, 5 + 2 * g);
         if (g + 1 >= ECL_MST_MAX_ROUNDS) { overflow = true; break; }
+        const bool guard = use_guard(P, L, __ldcg(&st->winners[g]));
         ++g;
-        passA(P, wl[cur], cnt, wl[cur ^ 1], &s_out);
+        passA(P, S, wl[cur ^ 1], &s_out, guard);
         cur ^= 1;
         __syncthreads();
-        cnt = s_out;
-        if (tid == 0 && cnt) atomicAdd(reinterpret_cast<unsigned long long*>(&st->live[g]), (unsigned long long)cnt);
+        S = compact_src(wl[cur], s_out);
+        if (tid == 0 && S.cnt) atomicAdd(reinterpret_cast<unsigned long long*>(&st->live[g]), (unsigned long long)S.cnt);
         trace_cta(P, 4 + 2 * g);
         grid.sync();
         stamp(P, 4 + 2 * g);
@@ -631,7 +722,8 @@ static int fail(int code, const char* fmt, ...) {
 
 struct DevInfo {
     int sms = 0;
-    int occ = 0;
+    int occ = 0;       // resident k_rounds CTAs per SM
+    int pop_occ = 0;   // resident k_populate CTAs per SM
 };
 
 static std::mutex g_dev_mu;
@@ -648,6 +740,9 @@ static int device_info(DevInfo* out) {
         e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
         if (e == cudaSuccess) e = cudaDeviceGetAttribute(&coop, cudaDevAttrCooperativeLaunch, dev);
         if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_rounds<1>, kBlock, 0);
+        int pop_occ = 0;
+        if (e == cudaSuccess) e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&pop_occ, k_populate<1>, kPopBlock, 0);
+        g_dev[dev].pop_occ = pop_occ > 0 ? pop_occ : 1;
         if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "device query: %s", cudaGetErrorString(e));
         if (!coop || occ < 1) return fail(ECL_MST_ERR_CUDA, "cooperative launch unsupported (coop=%d occ=%d)", coop, occ);
         g_dev[dev].sms = sms;
@@ -720,9 +815,20 @@ int ecl_mst_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t* n
     if (G > nchunks) G = nchunks;                 // small graphs: fewer, fuller arenas
     if (G > kMaxGrid) G = kMaxGrid;
     if (G < 1) G = 1;
-    const long long cap = ceil_div(nchunks, G) * kChunk;
+    // populate: one pass of the GPU, every warp a region; W a multiple of G
+    // so that every k_rounds CTA starts from the same number of regions
+    long long W = (long long)di.sms * di.pop_occ * kPopWarps;
+    if (W > nchunks) W = nchunks;
+    if (W > kMaxPopWarps) W = kMaxPopWarps;
+    if (W > G * kMaxRegionsPerCta) W = G * kMaxRegionsPerCta;
+    W = std::max<long long>(1, W / G) * G;
+    const long long rcap = ceil_div(nchunks, W) * kChunk;
+    if (W * rcap > L.wl_cap) return fail(ECL_MST_ERR_WORKSPACE, "internal: regions exceed worklist capacity");
+    // k_rounds arenas: the worklist of CTA b never exceeds its first input,
+    // the W / G regions b, b + G, ...  (arenas in wl0 overlay the regions;
+    // they are first written after every CTA has consumed its regions)
+    const long long cap = (W / G) * rcap;
     if (cap >= (1LL << 30)) return fail(ECL_MST_ERR_TOO_LARGE, "arena of %lld tuples too large", cap);
-    if (G * cap > L.wl_cap) return fail(ECL_MST_ERR_WORKSPACE, "internal: arenas exceed worklist capacity");
 
     Params P;
     P.n = n;
@@ -730,6 +836,8 @@ int ecl_mst_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t* n
     P.nchunks = nchunks;
     P.G = (int)G;
     P.cap = cap;
+    P.W = (int)W;
+    P.rcap = rcap;
     P.nindex = reinterpret_cast<const long long*>(nindex);
     P.nlist = nlist;
     P.eweight = eweight;
@@ -739,6 +847,7 @@ int ecl_mst_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t* n
     P.in = reinterpret_cast<Internal*>(ws + L.internal);
     P.trace = o.trace ? reinterpret_cast<long long*>(ws + L.trace) : nullptr;
     P.rowstart = reinterpret_cast<int*>(ws + L.rowstart);
+    P.region = reinterpret_cast<int4*>(ws + L.region);
     P.key = reinterpret_cast<long long*>(ws + L.key);
     P.parent = reinterpret_cast<int*>(ws + L.parent);
     P.wl0 = reinterpret_cast<int4*>(ws + L.wl0);
@@ -755,7 +864,7 @@ int ecl_mst_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t* n
         return fail(ECL_MST_ERR_INVALID, "nlist/eweight must be 16-byte and in_mst 4-byte aligned");
 
     const long long init_blocks = std::min<long long>(ceil_div((long long)n, 256), (long long)di.sms * 8);
-    const long long pop_blocks = ceil_div(nchunks, kPopWarps);
+    const long long pop_blocks = ceil_div(W, kPopWarps);
     if (pop_blocks > INT_MAX) return fail(ECL_MST_ERR_TOO_LARGE, "too many populate CTAs");
     void* args[] = {&P};
     cudaError_t e = cudaMemsetAsync(P.st, 0, sizeof(ecl_mst_stats), s);
@@ -767,7 +876,8 @@ int ecl_mst_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t* n
     if (e == cudaSuccess)
         e = cudaLaunchCooperativeKernel(reinterpret_cast<const void*>(k_rounds<1>), dim3((unsigned)G), dim3(kBlock), args, 0, s);
     if (e == cudaSuccess) {
-        k_flatten<<<(unsigned)std::max<long long>(init_blocks, 1), 256, 0, s>>>(P);
+        k_flatten<1><<<(unsigned)std::max<long long>(init_blocks, 1), 256, 0, s>>>(P);
+        k_flatten<2><<<(unsigned)std::max<long long>(init_blocks, 1), 256, 0, s>>>(P);
         k_populate<2><<<(unsigned)pop_blocks, kPopBlock, 0, s>>>(P);
         e = cudaGetLastError();
     }

@@ -11,8 +11,12 @@ import sys
 def main():
     rep = sys.argv[1]
     top = int(sys.argv[2]) if len(sys.argv) > 2 else 40
-    out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source=cuda,sass"],
-                         capture_output=True, text=True).stdout
+    cmd = ["ncu", "-i", rep, "--page", "source", "--csv", "--print-source=cuda,sass"]
+    if len(sys.argv) > 3:
+        cmd += ["--kernel-name", sys.argv[3]]
+    if len(sys.argv) > 4:
+        cmd += ["--launch-skip", sys.argv[4], "--launch-count", "1"]
+    out = subprocess.run(cmd, capture_output=True, text=True).stdout
     rows = list(csv.reader(io.StringIO(out)))
     cur_file = "?"
     hdr = None
