@@ -30,8 +30,12 @@ import torch  # noqa: E402
 
 PEAKS_FILE = os.path.join(ROOT, "MEASURED_PEAKS.json")
 PROFILE_SUMMARY = os.path.join(ROOT, "profiles", "ncu_summary_latest.json")
+LAUNCHES_PER_STEP = 8   # k_init, k_populate<1>, k_rounds<1>, k_flatten<1>, k_flatten<2>, k_populate<2>, k_rounds<2>, k_finalize
 CONFIG_NAMES = {"grid": "C1", "road": "C2", "rgg": "C3", "rmat": "C4", "uniform": "C5"}
 METRIC = "MSF edges/sec and ms/graph"
+KERNEL_OF_STAGE = {"init": "k_init", "populate1": "k_populate<1>", "rounds1": "k_rounds<1>",
+                   "flatten": "k_flatten<1,2>", "populate2": "k_populate<2>", "rounds2": "k_rounds<2>",
+                   "finalize": "k_finalize"}
 
 
 def parse():
@@ -116,31 +120,31 @@ class ClockSampler:
 
 
 def algorithmic_bytes(n: int, M: int, st: dict) -> dict:
-    """Bytes the method must move per launch.
+    """Bytes the method must move per launch, by kernel stage.
 
-    init        12 B/vertex  (parent 4 + best-edge key 8)
+    init        20 B/vertex  (nindex 8 read; parent 4 + best-edge key 8 written)
     populate    8 B/CSR entry (nlist+eweight) + 8 B/vertex (nindex) [+1 B/entry in_mst, phase 1]
                 + per emitted tuple 16 B write + 2x8 B key atomicMin
-                [phase 2: + 2x4 B parent gathers per heavy canonical edge, + 8 B/vertex flatten]
-    pass A      per input tuple 16 B read + 2x4 B parent; per survivor 16 B write + 2x8 B key min
-    pass B      per tuple 16 B read + 2x8 B key reads; per winner 4 B hook + 8 B key reset + 1 B mark
+                [phase 2: + 2x4 B parent gathers per heavy canonical edge]
+    flatten     8 B/vertex (parent read + write)
+    rounds      pass A: per input tuple 16 B read + 2x4 B parent; per survivor 16 B write + 2x8 B key min
+                pass B: per tuple 16 B read + 2x8 B key reads; per winner 4 B hook + 8 B key reset + 1 B mark
     """
     live = st["live"]
     win = st["winners"]
     R = len(live)
     p2 = st["phase2_round"]
-    b = {"init": 12 * n}
-    b["populate"] = (8 * M + 8 * n + M) + 32 * (live[0] if R else 0)
-    passA = passB = 0
-    for g in range(1, R):
-        if g == p2:
-            b["populate"] += 8 * M + 16 * n + 8 * st["heavy_edges"] + 32 * live[g]
-            continue
-        passA += 24 * live[g - 1] + 32 * live[g]
+    b = {"init": 20 * n, "populate1": 0, "rounds1": 0, "flatten": 0, "populate2": 0, "rounds2": 0}
     for g in range(R):
-        passB += 32 * live[g] + 13 * win[g]
-    b["passA"] = passA
-    b["passB"] = passB
+        ph = "2" if (p2 >= 0 and g >= p2) else "1"
+        if g == 0:
+            b["populate1"] += 8 * M + 8 * n + M + 32 * live[0]
+        elif g == p2:
+            b["flatten"] += 8 * n
+            b["populate2"] += 8 * M + 8 * n + 8 * st["heavy_edges"] + 32 * live[g]
+        else:
+            b["rounds" + ph] += 24 * live[g - 1] + 32 * live[g]
+        b["rounds" + ph] += 32 * live[g] + 13 * win[g]
     b["total"] = sum(b.values())
     return b
 
@@ -264,6 +268,7 @@ def main():
     stream = torch.cuda.current_stream()
     opt_kw = {k: int(v) for k, v in (o.split("=", 1) for o in args.opt)}
     opts = eclmst.default_options(**opt_kw)
+    opts.trace |= 2     # CUDA events between the library's kernels (per-kernel roofline)
 
     def step():
         eclmst.ecl_mst_device(n, g.nindex, g.nlist, g.eweight, in_mst_out=in_mst, total_weight_out=total,
@@ -281,11 +286,13 @@ def main():
         torch.distributed.barrier()
     torch.cuda.synchronize()
     wall0 = time.perf_counter()
+    kern = []
     for i in range(args.steps):
         flush.zero_()                      # L2 flush between timed steps (outside the events)
         ev[i][0].record(stream)
         step()
         ev[i][1].record(stream)
+        kern.append(eclmst.ecl_mst_kernel_times())   # waits for this step's events
     torch.cuda.synchronize()
     if world > 1:
         torch.distributed.barrier()
@@ -351,11 +358,13 @@ def main():
 
     peak, peak_src = load_peaks()
     ab = algorithmic_bytes(n, M, st)
-    achieved = ab["total"] / (ms / 1e3) / 1e9
+    kern_ms = {k: sum(d[k] for d in kern) / len(kern) for k in kern[0]}
+    dominant = max(("populate1", "rounds1", "populate2", "rounds2", "init", "flatten"), key=lambda k: kern_ms[k])
+    achieved = ab[dominant] / (kern_ms[dominant] / 1e3) / 1e9
     prof = load_traffic()
     traffic = None
     if prof and prof.get("workload") == g.name:
-        traffic = prof.get("dram_bytes_per_launch")
+        traffic = prof.get("dram_bytes_per_launch", {}).get(dominant)
     value = world * M / (ms_max / 1e3)
     line = {
         "metric": METRIC, "value": value, "unit": "edges/s", "n_gpus": world, "steps": args.steps,
@@ -368,11 +377,17 @@ def main():
                          "between steps"},
         "ms_per_graph": ms_max, "ms_per_step_all": per_step, "wall_s": wall,
         "edges_per_s_undirected": world * st["canonical_edges"] / (ms_max / 1e3),
-        "gpu_launches": args.steps,
+        "gpu_launches": args.steps * LAUNCHES_PER_STEP,
         "clocks": clocks,
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
-                     "kernel": "mst_persistent", "algorithmic_bytes": ab},
+                     "kernel": KERNEL_OF_STAGE[dominant], "stage": dominant,
+                     "kernel_share_of_step": kern_ms[dominant] / ms,
+                     "algorithmic_bytes_per_launch": ab[dominant],
+                     "whole_step": {"algorithmic_bytes": ab["total"],
+                                    "achieved_gbs": ab["total"] / (ms / 1e3) / 1e9,
+                                    "frac": ab["total"] / (ms / 1e3) / 1e9 / peak},
+                     "stage_ms": kern_ms, "stage_bytes": ab},
         "cpu_baseline": cpu_baseline,
         "e2e": e2e,
         "parity_vs_oracle": parity,

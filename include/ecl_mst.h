@@ -67,7 +67,8 @@ typedef struct ecl_mst_options {
                                 slots are still mostly inf and the guard only adds latency */
     int32_t flatten;         /* 1 (default) compress every path once before the phase-2 populate; 0 off */
     int32_t max_ctas;        /* 0 = fill the GPU (SMs x resident CTAs); else cap the grid */
-    int32_t trace;           /* 1: record every CTA's end time of every stage (ecl_mst_read_trace) */
+    int32_t trace;           /* bit 0: record every CTA's end time of every stage (ecl_mst_read_trace);
+                                bit 1: CUDA events between the kernels (ecl_mst_kernel_times) */
     uint64_t seed;           /* seed of the threshold sample */
 } ecl_mst_options;
 
@@ -137,6 +138,13 @@ int64_t ecl_mst(int32_t n, const int64_t *nindex, const int32_t *nlist,
  * ECL_MST_ERR_*. */
 #define ECL_MST_TRACE_CTAS 4096
 int ecl_mst_read_trace(const void *workspace, int64_t *out, size_t max_entries, void *stream);
+
+/* Diagnostics: after a call with opts.trace & 2 on this thread, waits for it
+ * and writes the device time (ms, CUDA events on the call's stream) of its
+ * stages to ms_out: [0] memset+init, [1] populate phase 1, [2] rounds phase 1,
+ * [3] flatten, [4] populate phase 2, [5] rounds phase 2, [6] finalize.
+ * Returns the number of values written (<= max_stages) or ECL_MST_ERR_*. */
+int ecl_mst_kernel_times(float *ms_out, int32_t max_stages);
 
 /* Frees the device buffers cached by ecl_mst(). */
 void ecl_mst_release_host_cache(void);

@@ -17,6 +17,7 @@ from ._native import (  # noqa: F401
     ecl_mst_device,
     ecl_mst_read_stats,
     ecl_mst_read_trace,
+    ecl_mst_kernel_times,
     ecl_mst_release_host_cache,
     ecl_mst_workspace_bytes,
     lib_path,
@@ -24,7 +25,7 @@ from ._native import (  # noqa: F401
 )
 
 __all__ = [
-    "ecl_mst", "ecl_mst_device", "ecl_mst_read_stats", "ecl_mst_read_trace", "ecl_mst_workspace_bytes",
+    "ecl_mst", "ecl_mst_device", "ecl_mst_read_stats", "ecl_mst_read_trace", "ecl_mst_kernel_times", "ecl_mst_workspace_bytes",
     "ecl_mst_release_host_cache", "default_options", "EclMstError", "EclMstOptions",
     "EclMstStats", "load", "lib_path", "EXPORTED",
 ]

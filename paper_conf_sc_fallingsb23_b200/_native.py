@@ -68,7 +68,8 @@ _lib = None
 
 
 def lib_path() -> str:
-    return _build.LIB
+    # ECLMST_LIB: load an alternative build of the same library (A/B experiments)
+    return os.environ.get("ECLMST_LIB", _build.LIB)
 
 
 def load(build_if_missing: bool = False):
@@ -76,12 +77,13 @@ def load(build_if_missing: bool = False):
     global _lib
     if _lib is not None:
         return _lib
-    if not os.path.exists(_build.LIB):
-        if not build_if_missing:
-            raise ImportError(f"libeclmst.so not built ({_build.LIB}); run `python -m "
+    path = lib_path()
+    if not os.path.exists(path):
+        if not build_if_missing or path != _build.LIB:
+            raise ImportError(f"libeclmst.so not built ({path}); run `python -m "
                               f"paper_conf_sc_fallingsb23_b200.build` or __graft_entry__.build()")
         _build.build()
-    L = ctypes.CDLL(_build.LIB)
+    L = ctypes.CDLL(path)
     vp, i32, i64, sz = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64, ctypes.c_size_t
     L.ecl_mst_abi_version.restype = ctypes.c_int
     L.ecl_mst_last_error.restype = ctypes.c_char_p
@@ -97,6 +99,8 @@ def load(build_if_missing: bool = False):
     L.ecl_mst_release_host_cache.restype = None
     L.ecl_mst_read_trace.restype = ctypes.c_int
     L.ecl_mst_read_trace.argtypes = [vp, vp, sz, vp]
+    L.ecl_mst_kernel_times.restype = ctypes.c_int
+    L.ecl_mst_kernel_times.argtypes = [vp, i32]
     if L.ecl_mst_abi_version() != 1:
         raise ImportError("libeclmst.so ABI version mismatch")
     _lib = L
@@ -105,7 +109,7 @@ def load(build_if_missing: bool = False):
 
 EXPORTED = ["ecl_mst_abi_version", "ecl_mst_last_error", "ecl_mst_default_options",
             "ecl_mst_workspace_bytes", "ecl_mst_device", "ecl_mst_read_stats", "ecl_mst",
-            "ecl_mst_release_host_cache", "ecl_mst_read_trace"]
+            "ecl_mst_release_host_cache", "ecl_mst_read_trace", "ecl_mst_kernel_times"]
 
 
 def _err(code):
@@ -215,6 +219,18 @@ def ecl_mst_read_trace(workspace, stats, stream=None):
     if rc != OK:
         _err(rc)
     return out.view(slots, TRACE_CTAS)[:, : stats["grid"]]
+
+
+KERNEL_STAGES = ["init", "populate1", "rounds1", "flatten", "populate2", "rounds2", "finalize"]
+
+
+def ecl_mst_kernel_times():
+    """Per-stage device times (ms) of the last call made with options.trace & 2."""
+    out = (ctypes.c_float * len(KERNEL_STAGES))()
+    rc = load().ecl_mst_kernel_times(out, len(KERNEL_STAGES))
+    if rc < 0:
+        _err(rc)
+    return dict(zip(KERNEL_STAGES, list(out)[:rc]))
 
 
 def ecl_mst(n, nindex, nlist, eweight, in_mst_out):

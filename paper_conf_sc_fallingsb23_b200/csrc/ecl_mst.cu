@@ -213,7 +213,10 @@ __global__ void __launch_bounds__(256) k_init(Params P) {
 // k_populate<PH>: one warp per 128-entry CSR chunk
 // ---------------------------------------------------------------------------
 template <int PH>
-__global__ void __launch_bounds__(kPopBlock, 8) k_populate(Params P) {
+#ifndef ECL_POP_MINB
+#define ECL_POP_MINB 4
+#endif
+__global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) {
     __shared__ int s_mark[kPopWarps][kChunk];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     if (PH == 2 && !phase2_needed(P)) return;
@@ -235,20 +238,11 @@ __global__ void __launch_bounds__(kPopBlock, 8) k_populate(Params P) {
     int4* const out = P.wl0 + (long long)w * P.rcap;
     int cnt = 0, canon_cnt = 0, heavy_cnt = 0;
     bool err = false;
-    for (long long c = w; c < P.nchunks; c += P.W) {
-    bool keep[kItems];
-    int4 t[kItems];
-#pragma unroll
-    for (int k = 0; k < kItems; ++k) keep[k] = false;
-    if (c < P.nchunks) {
+    const int p0 = lane * kItems;
+    // CSR entries of chunk c (lane owns entries p0 .. p0+3), streaming loads
+    auto load_entries = [&](long long c, int (&vv)[kItems], int (&ww)[kItems]) {
         const long long c0 = c * kChunk;
-        const long long c1 = min(c0 + (long long)kChunk, P.M);
-        const int len = (int)(c1 - c0);
-        const int p0 = lane * kItems;
-        // rows of this chunk: r0 = row of entry c0; rows r0+1 .. r_last start inside
-        const int r0 = __ldg(P.rowstart + c);
-        const int r_last = (c + 1 < P.nchunks) ? __ldg(P.rowstart + c + 1) : P.n - 1;
-        int vv[kItems], ww[kItems];
+        const int len = (int)(min(c0 + (long long)kChunk, P.M) - c0);
         if (p0 + kItems <= len) {
             const int4 a = __ldcs(reinterpret_cast<const int4*>(P.nlist + c0 + p0));
             const int4 b = __ldcs(reinterpret_cast<const int4*>(P.eweight + c0 + p0));
@@ -262,17 +256,51 @@ __global__ void __launch_bounds__(kPopBlock, 8) k_populate(Params P) {
                 ww[k] = ok ? __ldcs(P.eweight + c0 + p0 + k) : 0;
             }
         }
+    };
+    // software pipeline, one chunk ahead: the row bracket and the CSR entries
+    // of the next chunk are in flight while this one is processed (a deeper
+    // prefetch of the row starts measured no faster)
+    int nr0 = 0, nrl = 0, nv[kItems], nw[kItems];
+    if (w < P.nchunks) {
+        nr0 = __ldg(P.rowstart + w);
+        nrl = (w + 1 < P.nchunks) ? __ldg(P.rowstart + w + 1) : P.n - 1;
+        load_entries(w, nv, nw);
+    }
+    for (long long c = w; c < P.nchunks; c += P.W) {
+    bool keep[kItems];
+    int4 t[kItems];
+#pragma unroll
+    for (int k = 0; k < kItems; ++k) keep[k] = false;
+    {
+        const long long c0 = c * kChunk;
+        const long long c1 = min(c0 + (long long)kChunk, P.M);
+        const int len = (int)(c1 - c0);
+        // rows of this chunk: r0 = row of entry c0; rows r0+1 .. r_last start inside
+        const int r0 = nr0, r_last = nrl;
+        int vv[kItems], ww[kItems];
+#pragma unroll
+        for (int k = 0; k < kItems; ++k) {
+            vv[k] = nv[k];
+            ww[k] = nw[k];
+        }
+        const long long cn = c + P.W;
+        if (cn < P.nchunks) {
+            nr0 = __ldg(P.rowstart + cn);
+            nrl = (cn + 1 < P.nchunks) ? __ldg(P.rowstart + cn + 1) : P.n - 1;
+            load_entries(cn, nv, nw);
+        }
         int* mark = s_mark[warp];
 #pragma unroll
-        for (int i = lane; i < kChunk; i += 32) mark[i] = (i == 0) ? r0 : -1;
+        for (int i = lane; i < kChunk; i += 32) mark[i] = -1;
         __syncwarp();
-        for (int rb = r0 + 1; rb <= r_last; rb += 32) {
-            const int r = rb + lane;
-            if (r <= r_last) {
-                const long long s = P.nindex[r];
-                if (s >= c0 && s < c1) atomicMax(&mark[s - c0], r);
-                else if (s < c0) err = true;
-            }
+        for (int rb = r0 + 1; rb <= r_last; rb += 64) {   // two independent batches of row starts
+            const int ra = rb + lane, rz = rb + 32 + lane;
+            const long long sa = ra <= r_last ? __ldg(P.nindex + ra) : LLONG_MAX;
+            const long long sz = rz <= r_last ? __ldg(P.nindex + rz) : LLONG_MAX;
+            if (sa >= c0 && sa < c1) atomicMax(&mark[sa - c0], ra);
+            else if (sa < c0) err = true;
+            if (sz >= c0 && sz < c1) atomicMax(&mark[sz - c0], rz);
+            else if (sz < c0) err = true;
         }
         __syncwarp();
         int row[kItems];
@@ -288,9 +316,9 @@ __global__ void __launch_bounds__(kPopBlock, 8) k_populate(Params P) {
             if (lane >= o) incl = max(incl, y);
         }
         int excl = __shfl_up_sync(kFull, incl, 1);
-        if (lane == 0) excl = INT_MIN;
+        if (lane == 0) excl = r0;                 // position 0 belongs to row r0
 #pragma unroll
-        for (int k = 0; k < kItems; ++k) row[k] = max(row[k], excl);
+        for (int k = 0; k < kItems; ++k) row[k] = max(row[k], max(excl, r0));
 
         if (PH == 1) {   // every in_mst byte is written once, here (Alg. 1 "not in MST")
             if (p0 + kItems <= len) {
@@ -729,6 +757,15 @@ struct DevInfo {
 static std::mutex g_dev_mu;
 static DevInfo g_dev[64];
 
+// per-thread CUDA events bracketing the kernels of the last timed call
+constexpr int kTimedStages = 7;   // init, populate1, rounds1, flatten, populate2, rounds2, finalize
+struct Timing {
+    bool ready = false;
+    bool valid = false;
+    cudaEvent_t ev[kTimedStages + 1];
+};
+static thread_local Timing g_timing;
+
 static int device_info(DevInfo* out) {
     int dev = 0;
     cudaError_t e = cudaGetDevice(&dev);
@@ -867,28 +904,70 @@ int ecl_mst_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t* n
     const long long pop_blocks = ceil_div(W, kPopWarps);
     if (pop_blocks > INT_MAX) return fail(ECL_MST_ERR_TOO_LARGE, "too many populate CTAs");
     void* args[] = {&P};
-    cudaError_t e = cudaMemsetAsync(P.st, 0, sizeof(ecl_mst_stats), s);
+    // opts.trace bit 1: CUDA events between the kernels (ecl_mst_kernel_times)
+    const bool timing = (o.trace & 2) != 0;
+    if (timing && !g_timing.ready) {
+        for (int i = 0; i < kTimedStages + 1; ++i) {
+            cudaError_t e0 = cudaEventCreate(&g_timing.ev[i]);
+            if (e0 != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "cudaEventCreate: %s", cudaGetErrorString(e0));
+        }
+        g_timing.ready = true;
+    }
+    g_timing.valid = false;
+    int ev_i = 0;
+    auto mark = [&]() -> cudaError_t {
+        return timing ? cudaEventRecord(g_timing.ev[ev_i++], s) : cudaSuccess;
+    };
+    const unsigned flat_blocks = (unsigned)std::max<long long>(init_blocks, 1);
+    cudaError_t e = mark();
+    if (e == cudaSuccess) e = cudaMemsetAsync(P.st, 0, sizeof(ecl_mst_stats), s);
     if (e == cudaSuccess) {
-        k_init<<<(unsigned)std::max<long long>(init_blocks, 1), 256, 0, s>>>(P);
+        k_init<<<flat_blocks, 256, 0, s>>>(P);
+        e = cudaGetLastError();
+    }
+    if (e == cudaSuccess) e = mark();
+    if (e == cudaSuccess) {
         k_populate<1><<<(unsigned)pop_blocks, kPopBlock, 0, s>>>(P);
         e = cudaGetLastError();
     }
+    if (e == cudaSuccess) e = mark();
     if (e == cudaSuccess)
         e = cudaLaunchCooperativeKernel(reinterpret_cast<const void*>(k_rounds<1>), dim3((unsigned)G), dim3(kBlock), args, 0, s);
+    if (e == cudaSuccess) e = mark();
     if (e == cudaSuccess) {
-        k_flatten<1><<<(unsigned)std::max<long long>(init_blocks, 1), 256, 0, s>>>(P);
-        k_flatten<2><<<(unsigned)std::max<long long>(init_blocks, 1), 256, 0, s>>>(P);
+        k_flatten<1><<<flat_blocks, 256, 0, s>>>(P);
+        k_flatten<2><<<flat_blocks, 256, 0, s>>>(P);
+        e = cudaGetLastError();
+    }
+    if (e == cudaSuccess) e = mark();
+    if (e == cudaSuccess) {
         k_populate<2><<<(unsigned)pop_blocks, kPopBlock, 0, s>>>(P);
         e = cudaGetLastError();
     }
+    if (e == cudaSuccess) e = mark();
     if (e == cudaSuccess)
         e = cudaLaunchCooperativeKernel(reinterpret_cast<const void*>(k_rounds<2>), dim3((unsigned)G), dim3(kBlock), args, 0, s);
+    if (e == cudaSuccess) e = mark();
     if (e == cudaSuccess) {
         k_finalize<<<1, 32, 0, s>>>(P);
         e = cudaGetLastError();
     }
+    if (e == cudaSuccess) e = mark();
+    if (e == cudaSuccess && timing) g_timing.valid = true;
     if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "launch (G=%lld): %s", G, cudaGetErrorString(e));
     return ECL_MST_OK;
+}
+
+int ecl_mst_kernel_times(float* ms_out, int32_t max_stages) {
+    g_last_error.clear();
+    if (!ms_out) return fail(ECL_MST_ERR_INVALID, "null argument");
+    if (!g_timing.valid) return fail(ECL_MST_ERR_INVALID, "no timed run on this thread (opts.trace & 2)");
+    cudaError_t e = cudaEventSynchronize(g_timing.ev[kTimedStages]);
+    int n = 0;
+    for (; e == cudaSuccess && n < kTimedStages && n < max_stages; ++n)
+        e = cudaEventElapsedTime(&ms_out[n], g_timing.ev[n], g_timing.ev[n + 1]);
+    if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "kernel_times: %s", cudaGetErrorString(e));
+    return n;
 }
 
 int ecl_mst_read_stats(const void* workspace, ecl_mst_stats* out, void* stream) {

@@ -25,38 +25,56 @@ UNIT_SCALE = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12
               "nsecond": 1e-9}
 
 
+def stage_of(kernel_name):
+    k = kernel_name
+    for pat, st in (("k_init", "init"), ("k_populate<1>", "populate1"), ("k_populate<(int)1>", "populate1"),
+                    ("k_populate<2>", "populate2"), ("k_populate<(int)2>", "populate2"),
+                    ("k_rounds<1>", "rounds1"), ("k_rounds<(int)1>", "rounds1"),
+                    ("k_rounds<2>", "rounds2"), ("k_rounds<(int)2>", "rounds2"),
+                    ("k_flatten", "flatten"), ("k_finalize", "finalize")):
+        if pat in k:
+            return st
+    return k
+
+
 def full(rep, out, workload=None):
     raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
     rows = [r for r in csv.reader(io.StringIO(raw))]
     hdr, units = rows[0], rows[1]
-    kernels = []
+    per_stage = {}
     for vals in rows[2:]:
         d = {}
         for h, u, v in zip(hdr, units, vals):
             if h in FULL_METRICS or h == "Kernel Name":
                 try:
-                    x = float(v.replace(",", ""))
-                    d[h] = {"value": x, "unit": u}
+                    d[h] = {"value": float(v.replace(",", "")), "unit": u}
                 except ValueError:
                     d[h] = v
-        kernels.append(d)
-    k = kernels[0]
 
-    def si(name):
-        e = k.get(name)
-        if not isinstance(e, dict):
-            return None
-        return e["value"] * UNIT_SCALE.get(e["unit"], 1)
-    rd, wr, t = si("dram__bytes_read.sum"), si("dram__bytes_write.sum"), si("gpu__time_duration.sum")
-    summary = {
-        "report": rep, "workload": workload, "kernel": k.get("Kernel Name"),
-        "duration_s": t, "dram_read_bytes": rd, "dram_write_bytes": wr,
-        "dram_bytes_per_launch": (rd or 0) + (wr or 0),
-        "dram_gbs": ((rd or 0) + (wr or 0)) / t / 1e9 if t else None,
-        "metrics": {h: k[h] for h in FULL_METRICS if h in k},
-    }
+        def si(name):
+            e = d.get(name)
+            if not isinstance(e, dict):
+                return 0.0
+            return e["value"] * UNIT_SCALE.get(e["unit"], 1)
+        st = stage_of(d.get("Kernel Name", "?"))
+        e = per_stage.setdefault(st, {"kernel": d.get("Kernel Name"), "launches": 0, "duration_s": 0.0,
+                                      "dram_read_bytes": 0.0, "dram_write_bytes": 0.0, "metrics": []})
+        e["launches"] += 1
+        e["duration_s"] += si("gpu__time_duration.sum")
+        e["dram_read_bytes"] += si("dram__bytes_read.sum")
+        e["dram_write_bytes"] += si("dram__bytes_write.sum")
+        e["metrics"].append({h: d[h] for h in FULL_METRICS if h in d})
+    for e in per_stage.values():
+        e["dram_bytes"] = e["dram_read_bytes"] + e["dram_write_bytes"]
+        e["dram_gbs"] = e["dram_bytes"] / e["duration_s"] / 1e9 if e["duration_s"] else None
+    summary = {"report": rep, "workload": workload,
+               "note": "ncu --set full, one launch of every kernel of one MSF (cold L2, serialised replays)",
+               "dram_bytes_per_launch": {k: v["dram_bytes"] for k, v in per_stage.items()},
+               "stages": per_stage}
     json.dump(summary, open(out, "w"), indent=1)
-    print(json.dumps({x: summary[x] for x in ("kernel", "duration_s", "dram_bytes_per_launch", "dram_gbs")}))
+    for k, v in per_stage.items():
+        print(f"{k:10s} {v['duration_s']*1e3:8.3f} ms  dram {v['dram_bytes']/1e9:7.3f} GB  "
+              f"{(v['dram_gbs'] or 0):7.1f} GB/s")
 
 
 def launches(path, out):
