@@ -70,6 +70,9 @@ typedef struct ecl_mst_options {
     int32_t trace;           /* bit 0: record every CTA's end time of every stage (ecl_mst_read_trace);
                                 bit 1: CUDA events between the kernels (ecl_mst_kernel_times) */
     uint64_t seed;           /* seed of the threshold sample */
+    int32_t threshold_samples; /* sample size S for threshold_mode 0 (paper: 20; default
+                                  1024 -- same target, far less variance; <= 4096) */
+    int32_t reserved;
 } ecl_mst_options;
 
 /* per-run statistics written by the device into the workspace */
@@ -145,6 +148,47 @@ int ecl_mst_read_trace(const void *workspace, int64_t *out, size_t max_entries, 
  * [3] flatten, [4] populate phase 2, [5] rounds phase 2, [6] finalize.
  * Returns the number of values written (<= max_stages) or ECL_MST_ERR_*. */
 int ecl_mst_kernel_times(float *ms_out, int32_t max_stages);
+
+/* ------------------------------------------------------------------------
+ * Edge-sharded multi-GPU path (BASELINE.json north_star).
+ * One process per GPU.  Every rank passes the SAME full CSR (replicated,
+ * read-only); shard s of P = world * local_shards owns the 128-entry CSR
+ * chunks s, s + P, s + 2P, ... and the worklist tuples they produce.  Per
+ * round: local pass A over the rank's tuples -> ncclAllReduce(min, int64)
+ * of the n best-edge keys -> a set-centric pass B that every rank applies
+ * identically to its replicated union-find (a set with a finite key hooks
+ * along that edge; id -> (row, nlist[id]) through the replicated CSR).
+ * Output: every rank writes the full in_mst and the total weight.
+ * NCCL is the process's libnccl.so.2 (dlopen; torch's when torch is loaded,
+ * override with $ECLMST_NCCL_LIB).  The round loop is host-driven with one
+ * 8-byte device-to-host read per round (the termination test).
+ * ------------------------------------------------------------------------ */
+
+/* 128-byte NCCL unique id for ecl_mst_dist_init (create on one rank, broadcast). */
+int ecl_mst_dist_unique_id(void *uid_out);
+
+/* Creates a handle.  world > 1 needs uid (NCCL communicator of `world` ranks,
+ * this one `rank`, on the current device).  world == 1 with uid == NULL runs
+ * without NCCL; world == 1 with a uid builds a one-rank communicator. */
+int ecl_mst_dist_init(const void *uid, int32_t rank, int32_t world, void **handle_out);
+
+int ecl_mst_dist_finalize(void *handle);
+
+/* Number of CSR chunks shard `shard` of `nshards` owns (host helper). */
+int64_t ecl_mst_dist_shard_chunks(int64_t M, int32_t shard, int32_t nshards);
+
+/* Workspace bytes of ecl_mst_dist_device for one rank holding local_shards
+ * shards of a world of `world` ranks; 0 if too large. */
+size_t ecl_mst_dist_workspace_bytes(int64_t n, int64_t M, int32_t local_shards, int32_t world);
+
+/* The sharded hot path; arguments as ecl_mst_device.  local_shards > 1 (only
+ * with world == 1) runs that many virtual shards on this GPU with an
+ * on-device min-reduction in place of the allreduce -- the same algorithm
+ * and data flow, testable on one GPU.  Synchronises `stream` once per round. */
+int ecl_mst_dist_device(void *handle, int32_t local_shards, int32_t n, int64_t M,
+                        const int64_t *nindex, const int32_t *nlist, const int32_t *eweight,
+                        uint8_t *in_mst_out, int64_t *total_weight_out, void *workspace,
+                        size_t workspace_bytes, const ecl_mst_options *opts, void *stream);
 
 /* Frees the device buffers cached by ecl_mst(). */
 void ecl_mst_release_host_cache(void);

@@ -15,6 +15,12 @@ from ._native import (  # noqa: F401
     default_options,
     ecl_mst,
     ecl_mst_device,
+    ecl_mst_dist_device,
+    ecl_mst_dist_finalize,
+    ecl_mst_dist_init,
+    ecl_mst_dist_shard_chunks,
+    ecl_mst_dist_unique_id,
+    ecl_mst_dist_workspace_bytes,
     ecl_mst_read_stats,
     ecl_mst_read_trace,
     ecl_mst_kernel_times,
@@ -27,5 +33,8 @@ from ._native import (  # noqa: F401
 __all__ = [
     "ecl_mst", "ecl_mst_device", "ecl_mst_read_stats", "ecl_mst_read_trace", "ecl_mst_kernel_times", "ecl_mst_workspace_bytes",
     "ecl_mst_release_host_cache", "default_options", "EclMstError", "EclMstOptions",
-    "EclMstStats", "load", "lib_path", "EXPORTED",
+    "EclMstStats", "load", "lib_path", "EXPORTED", "ecl_mst_dist_device", "ecl_mst_dist_init",
+    "ecl_mst_dist_finalize", "ecl_mst_dist_shard_chunks", "ecl_mst_dist_unique_id",
+    "ecl_mst_dist_workspace_bytes", "dist",
 ]
+from . import dist  # noqa: E402,F401

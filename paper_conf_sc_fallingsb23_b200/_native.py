@@ -35,6 +35,8 @@ class EclMstOptions(ctypes.Structure):
         ("max_ctas", ctypes.c_int32),
         ("trace", ctypes.c_int32),
         ("seed", ctypes.c_uint64),
+        ("threshold_samples", ctypes.c_int32),
+        ("reserved", ctypes.c_int32),
     ]
 
 
@@ -101,6 +103,19 @@ def load(build_if_missing: bool = False):
     L.ecl_mst_read_trace.argtypes = [vp, vp, sz, vp]
     L.ecl_mst_kernel_times.restype = ctypes.c_int
     L.ecl_mst_kernel_times.argtypes = [vp, i32]
+    L.ecl_mst_dist_unique_id.restype = ctypes.c_int
+    L.ecl_mst_dist_unique_id.argtypes = [vp]
+    L.ecl_mst_dist_init.restype = ctypes.c_int
+    L.ecl_mst_dist_init.argtypes = [vp, i32, i32, ctypes.POINTER(ctypes.c_void_p)]
+    L.ecl_mst_dist_finalize.restype = ctypes.c_int
+    L.ecl_mst_dist_finalize.argtypes = [vp]
+    L.ecl_mst_dist_shard_chunks.restype = i64
+    L.ecl_mst_dist_shard_chunks.argtypes = [i64, i32, i32]
+    L.ecl_mst_dist_workspace_bytes.restype = sz
+    L.ecl_mst_dist_workspace_bytes.argtypes = [i64, i64, i32, i32]
+    L.ecl_mst_dist_device.restype = ctypes.c_int
+    L.ecl_mst_dist_device.argtypes = [vp, i32, i32, i64, vp, vp, vp, vp, vp, vp, sz,
+                                      ctypes.POINTER(EclMstOptions), vp]
     if L.ecl_mst_abi_version() != 1:
         raise ImportError("libeclmst.so ABI version mismatch")
     _lib = L
@@ -109,7 +124,9 @@ def load(build_if_missing: bool = False):
 
 EXPORTED = ["ecl_mst_abi_version", "ecl_mst_last_error", "ecl_mst_default_options",
             "ecl_mst_workspace_bytes", "ecl_mst_device", "ecl_mst_read_stats", "ecl_mst",
-            "ecl_mst_release_host_cache", "ecl_mst_read_trace", "ecl_mst_kernel_times"]
+            "ecl_mst_release_host_cache", "ecl_mst_read_trace", "ecl_mst_kernel_times",
+            "ecl_mst_dist_unique_id", "ecl_mst_dist_init", "ecl_mst_dist_finalize",
+            "ecl_mst_dist_shard_chunks", "ecl_mst_dist_workspace_bytes", "ecl_mst_dist_device"]
 
 
 def _err(code):
@@ -219,6 +236,71 @@ def ecl_mst_read_trace(workspace, stats, stream=None):
     if rc != OK:
         _err(rc)
     return out.view(slots, TRACE_CTAS)[:, : stats["grid"]]
+
+
+# ---- edge-sharded multi-GPU path ----
+
+def ecl_mst_dist_unique_id() -> bytes:
+    """128-byte NCCL unique id (create on one rank, broadcast to the others)."""
+    buf = ctypes.create_string_buffer(128)
+    rc = load().ecl_mst_dist_unique_id(buf)
+    if rc != OK:
+        _err(rc)
+    return buf.raw
+
+
+def ecl_mst_dist_init(uid, rank: int, world: int):
+    """Handle for ecl_mst_dist_device (uid None: world 1 without NCCL)."""
+    h = ctypes.c_void_p()
+    ubuf = ctypes.create_string_buffer(bytes(uid), 128) if uid is not None else None
+    rc = load().ecl_mst_dist_init(ubuf, int(rank), int(world), ctypes.byref(h))
+    if rc != OK:
+        _err(rc)
+    return h
+
+
+def ecl_mst_dist_finalize(handle):
+    load().ecl_mst_dist_finalize(handle)
+
+
+def ecl_mst_dist_shard_chunks(M: int, shard: int, nshards: int) -> int:
+    return int(load().ecl_mst_dist_shard_chunks(int(M), int(shard), int(nshards)))
+
+
+def ecl_mst_dist_workspace_bytes(n: int, M: int, local_shards: int = 1, world: int = 1) -> int:
+    b = load().ecl_mst_dist_workspace_bytes(int(n), int(M), int(local_shards), int(world))
+    if b == 0:
+        raise EclMstError(ERR_TOO_LARGE, f"graph too large (n={n}, M={M})")
+    return int(b)
+
+
+def ecl_mst_dist_device(handle, n, nindex, nlist, eweight, local_shards=1, world=1, in_mst_out=None,
+                        total_weight_out=None, workspace=None, options=None, stream=None):
+    """Sharded hot path on this rank's GPU (full replicated CSR in, full mask out)."""
+    dev = nlist.device
+    if dev.type != "cuda":
+        raise ValueError("ecl_mst_dist_device needs CUDA tensors (no CPU fallback)")
+    _check(nindex, torch.int64, "nindex", dev)
+    _check(nlist, torch.int32, "nlist", dev)
+    _check(eweight, torch.int32, "eweight", dev)
+    n = int(n)
+    M = int(nlist.numel())
+    if in_mst_out is None:
+        in_mst_out = torch.empty(M, dtype=torch.uint8, device=dev)
+    if total_weight_out is None:
+        total_weight_out = torch.empty(1, dtype=torch.int64, device=dev)
+    need = ecl_mst_dist_workspace_bytes(n, M, local_shards, world)
+    if workspace is None or workspace.numel() < need:
+        workspace = torch.empty(need, dtype=torch.uint8, device=dev)
+    opts = options if options is not None else default_options()
+    with torch.cuda.device(dev):
+        rc = load().ecl_mst_dist_device(handle, int(local_shards), n, M, nindex.data_ptr(), nlist.data_ptr(),
+                                        eweight.data_ptr(), in_mst_out.data_ptr(), total_weight_out.data_ptr(),
+                                        workspace.data_ptr(), workspace.numel(), ctypes.byref(opts),
+                                        _stream_ptr(stream))
+    if rc != OK:
+        _err(rc)
+    return in_mst_out, total_weight_out, workspace
 
 
 KERNEL_STAGES = ["init", "populate1", "rounds1", "flatten", "populate2", "rounds2", "finalize"]

@@ -38,9 +38,12 @@
 #include <cstdint>
 #include <cstdio>
 #include <cstring>
+#include <dlfcn.h>
+
 #include <algorithm>
 #include <mutex>
 #include <string>
+#include <vector>
 
 #include "device.cuh"
 #include "ecl_mst.h"
@@ -55,9 +58,11 @@ constexpr int kPopBlock = 32 * kPopWarps;
 constexpr int kMaxPopWarps = 65536;            // populate warps (= worklist regions), upper bound
 constexpr int kMaxRegionsPerCta = 256;         // regions a k_rounds CTA starts from
 constexpr int kTraceSlots = 2 * ECL_MST_MAX_ROUNDS + 4;
+constexpr int kMaxSamples = 4096;              // threshold sample size cap
 static_assert(kMaxGrid == ECL_MST_TRACE_CTAS, "trace layout");
 
 struct Internal {
+    unsigned long long reps;           // distributed path: sets with a finite key this round
     unsigned int done;                 // unused ticket
     int g_cur;                         // first global round of the running phase
     int g_end;                         // last global round of the finished phase
@@ -125,9 +130,19 @@ struct Params {
     int filter_mode;
     int threshold_mode;
     int threshold_value;
+    int samples;
     int halving;
     int guards;                       // -1 auto, 0 off, 1 on
     int flatten;
+    // edge sharding (distributed path; single GPU: shard 0 of 1)
+    int shard;                        // global shard id
+    int nshards;                      // total shards
+    long long nlocal;                 // chunks of this shard: shard, shard + nshards, ...
+    int zero_mst;                     // populate phase 1 zeroes its chunks of in_mst
+    int* acnt;                        // per arena tuple count (distributed pass A)
+    int* tgt;                         // per vertex hook target (distributed rep pass)
+    long long* const* keys_all;       // virtual shards: every shard's key array
+    int nkeys;
 };
 
 __device__ __forceinline__ void stamp(const Params& P, int slot) {
@@ -160,7 +175,11 @@ __global__ void __launch_bounds__(256) k_init(Params P) {
     bool err = false;
     for (long long v = i0; v < P.n; v += stride) {
         P.parent[v] = (int)v;                       // every vertex its own set
-        P.key[v] = kInf;                            // no minimum edge recorded
+        if (P.keys_all) {                           // no minimum edge recorded
+            for (int s2 = 0; s2 < P.nkeys; ++s2) P.keys_all[s2][v] = kInf;
+        } else {
+            P.key[v] = kInf;
+        }
         // chunk starts inside row v: rowstart[c] = v for c*kChunk in [s, e)
         const long long s = P.nindex[v], e = P.nindex[v + 1];
         if (e < s) err = true;
@@ -168,42 +187,44 @@ __global__ void __launch_bounds__(256) k_init(Params P) {
     }
     if (blockIdx.x == 0) {
         ecl_mst_stats* st = P.st;   // zeroed by a memset node just before this kernel
-        if (warp == 0) {
-            // filter decision (readings Q5-Q7)
-            const bool filtered = P.filter_mode < 0 ? (P.M >= 4LL * P.n) : (P.filter_mode != 0);
-            int T = INT_MAX;
-            if (filtered) {
-                if (P.threshold_mode == 1) {
-                    T = P.threshold_value;
-                } else {
-                    int w = INT_MAX;
-                    if (lane < 20) {
-                        const unsigned long long h = splitmix64(P.seed * 0x100000001B3ull + (unsigned long long)lane);
-                        w = P.eweight[(long long)(h % (unsigned long long)P.M)];
-                    }
-                    int rank = 0;
-                    for (int s = 0; s < 20; ++s) {
-                        const int ws = __shfl_sync(kFull, w, s);
-                        if (lane < 20 && (ws < w || (ws == w && s < lane))) ++rank;
-                    }
-                    long long kpos = (80LL * P.n) / P.M;   // c|V| lightest of M entries: 20 * 4n / M
-                    if (kpos > 19) kpos = 19;
-                    const unsigned b = __ballot_sync(kFull, lane < 20 && rank == (int)kpos);
-                    T = __shfl_sync(kFull, w, __ffs(b) - 1);
+        __shared__ int s_w[kMaxSamples];
+        __shared__ int s_T;
+        // filter decision (readings Q5-Q7): estimate the
+        // weight of the c|V| lightest of the M entries (c = 4) from S random
+        // entries: T = the sample of rank floor(S * 4n / M)
+        const bool filtered = P.filter_mode < 0 ? (P.M >= 4LL * P.n) : (P.filter_mode != 0);
+        if (tid == 0) s_T = (filtered && P.threshold_mode == 1) ? P.threshold_value : INT_MAX;
+        if (filtered && P.threshold_mode == 0) {
+            const int S = P.samples;
+            for (int i = tid; i < S; i += blockDim.x) {
+                const unsigned long long h = splitmix64(P.seed * 0x100000001B3ull + (unsigned long long)i);
+                s_w[i] = P.eweight[(long long)(h % (unsigned long long)P.M)];
+            }
+            __syncthreads();
+            long long kpos = ((long long)S * 4LL * P.n) / P.M;
+            if (kpos > S - 1) kpos = S - 1;
+            for (int i = tid; i < S; i += blockDim.x) {
+                const int wi = s_w[i];
+                int rank = 0;
+                for (int t = 0; t < S; ++t) {
+                    const int wt = s_w[t];
+                    rank += (wt < wi) || (wt == wi && t < i);
                 }
+                if (rank == (int)kpos) s_T = wi;
             }
-            if (lane == 0) {
-                st->t_ns[0] = (long long)globaltimer_ns();
-                st->filtered = filtered ? 1 : 0;
-                st->threshold = T;
-                st->grid = P.G;
-                st->block = kBlock;
-                st->phase2_round = -1;
-                if (P.nindex[0] != 0 || P.nindex[P.n] != P.M) err = true;
-                P.in->g_cur = 0;
-                P.in->g_end = 0;
-                P.in->done = 0;
-            }
+        }
+        __syncthreads();
+        if (tid == 0) {
+            st->t_ns[0] = (long long)globaltimer_ns();
+            st->filtered = filtered ? 1 : 0;
+            st->threshold = s_T;
+            st->grid = P.G;
+            st->block = kBlock;
+            st->phase2_round = -1;
+            if (P.nindex[0] != 0 || P.nindex[P.n] != P.M) err = true;
+            P.in->g_cur = 0;
+            P.in->g_end = 0;
+            P.in->done = 0;
         }
     }
     if (err) atomicExch(&P.st->status, ECL_MST_ERR_INPUT);
@@ -260,13 +281,17 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
     // software pipeline, one chunk ahead: the row bracket and the CSR entries
     // of the next chunk are in flight while this one is processed (a deeper
     // prefetch of the row starts measured no faster)
+    // (edge sharding: this shard owns chunks shard, shard + nshards, ...;
+    // lc indexes them, c is the global chunk)
     int nr0 = 0, nrl = 0, nv[kItems], nw[kItems];
-    if (w < P.nchunks) {
-        nr0 = __ldg(P.rowstart + w);
-        nrl = (w + 1 < P.nchunks) ? __ldg(P.rowstart + w + 1) : P.n - 1;
-        load_entries(w, nv, nw);
+    if (w < P.nlocal) {
+        const long long c = P.shard + (long long)w * P.nshards;
+        nr0 = __ldg(P.rowstart + c);
+        nrl = (c + 1 < P.nchunks) ? __ldg(P.rowstart + c + 1) : P.n - 1;
+        load_entries(c, nv, nw);
     }
-    for (long long c = w; c < P.nchunks; c += P.W) {
+    for (long long lc = w; lc < P.nlocal; lc += P.W) {
+    const long long c = P.shard + lc * P.nshards;
     bool keep[kItems];
     int4 t[kItems];
 #pragma unroll
@@ -283,8 +308,9 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
             vv[k] = nv[k];
             ww[k] = nw[k];
         }
-        const long long cn = c + P.W;
-        if (cn < P.nchunks) {
+        const long long lcn = lc + P.W;
+        const long long cn = P.shard + lcn * P.nshards;
+        if (lcn < P.nlocal) {
             nr0 = __ldg(P.rowstart + cn);
             nrl = (cn + 1 < P.nchunks) ? __ldg(P.rowstart + cn + 1) : P.n - 1;
             load_entries(cn, nv, nw);
@@ -320,7 +346,7 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
 #pragma unroll
         for (int k = 0; k < kItems; ++k) row[k] = max(row[k], max(excl, r0));
 
-        if (PH == 1) {   // every in_mst byte is written once, here (Alg. 1 "not in MST")
+        if (PH == 1 && P.zero_mst) {   // every in_mst byte is written once, here (Alg. 1 "not in MST")
             if (p0 + kItems <= len) {
                 __stcs(reinterpret_cast<unsigned*>(P.in_mst + c0 + p0), 0u);
             } else {
@@ -731,6 +757,161 @@ __global__ void k_finalize(Params P) {
     }
 }
 
+
+// ---------------------------------------------------------------------------
+// Distributed (edge-sharded) MSF -- SURVEY §8(e).  Every rank holds the full
+// CSR, a replicated union-find and a full key array; it owns the CSR chunks
+// c = shard, shard + P, ... and the tuples they produce.  Per round:
+//   allreduce(key, min) over the ranks  ->  every rank knows each set's
+//   lightest edge;  rep-centric pass B, identical on every rank (each set
+//   with a finite key hooks along its edge, looked up by id in the CSR);
+//   local pass A over the rank's own tuples.
+// ---------------------------------------------------------------------------
+
+// row of CSR entry j: binary search inside the rows of j's chunk
+__device__ __forceinline__ int row_of_entry(const Params& P, long long j) {
+    const long long c = j / kChunk;
+    int lo = __ldg(P.rowstart + c);
+    int hi = (c + 1 < P.nchunks) ? __ldg(P.rowstart + c + 1) : P.n - 1;
+    while (lo < hi) {   // largest r in [lo, hi] with nindex[r] <= j
+        const int mid = lo + ((hi - lo + 1) >> 1);
+        if (__ldg(P.nindex + mid) <= j) lo = mid;
+        else hi = mid - 1;
+    }
+    return lo;
+}
+
+// virtual shards on one GPU: the "allreduce" is an elementwise min over the
+// shards' key arrays, written back to every copy (as NCCL would)
+__global__ void __launch_bounds__(256) k_vreduce(Params P) {
+    const long long stride = (long long)gridDim.x * blockDim.x;
+    for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < P.n; v += stride) {
+        long long m = kInf;
+        for (int s2 = 0; s2 < P.nkeys; ++s2) m = min(m, P.keys_all[s2][v]);
+        for (int s2 = 0; s2 < P.nkeys; ++s2) P.keys_all[s2][v] = m;
+    }
+}
+
+// rep pass 1: for every set x with a finite (reduced) key, the other end's set
+// q of its lightest edge, and whether that edge is q's lightest too (mutual)
+__global__ void __launch_bounds__(256) k_dist_reps1(Params P) {
+    const long long stride = (long long)gridDim.x * blockDim.x;
+    unsigned long long found = 0;
+    for (long long x = (long long)blockIdx.x * blockDim.x + threadIdx.x; x < P.n; x += stride) {
+        const long long kx = P.key[x];
+        if (kx == kInf) continue;
+        ++found;
+        const unsigned j = (unsigned)(kx & 0xffffffffll);
+        const int u = row_of_entry(P, (long long)j);
+        const int v = __ldg(P.nlist + j);
+        const int pu = find_root(P.parent, u, false), pv = find_root(P.parent, v, false);
+        const int q = (pu == (int)x) ? pv : pu;
+        const bool mutual = P.key[q] == kx;
+        P.tgt[x] = q | (mutual ? (int)0x80000000 : 0);
+    }
+    found = warp_sum(found);
+    if ((threadIdx.x & 31) == 0 && found) atomicAdd(reinterpret_cast<unsigned long long*>(&P.in->reps), found);
+}
+
+// rep pass 2 (L30-31, L34-37): hook, mark, sum, reset -- the same rule as the
+// tuple-centric pass B, so the partition after each round is the same
+__global__ void __launch_bounds__(256) k_dist_reps2(Params P, int g) {
+    const long long stride = (long long)gridDim.x * blockDim.x;
+    long long wsum = 0, wcnt = 0;
+    for (long long x = (long long)blockIdx.x * blockDim.x + threadIdx.x; x < P.n; x += stride) {
+        const long long kx = P.key[x];
+        if (kx == kInf) continue;
+        const int t = P.tgt[x];
+        const int q = t & 0x7fffffff;
+        const bool mutual = t < 0;
+        if (!mutual || (int)x > q) P.parent[x] = q;
+        if (!mutual || (int)x < q) {
+            P.in_mst[(unsigned)(kx & 0xffffffffll)] = 1;
+            wsum += (int)(kx >> 32);
+            wcnt += 1;
+        }
+        for (int s2 = 0; s2 < P.nkeys; ++s2) P.keys_all[s2][x] = kInf;
+    }
+    wsum = warp_sum(wsum);
+    wcnt = warp_sum(wcnt);
+    if ((threadIdx.x & 31) == 0 && wcnt) {
+        atomicAdd(reinterpret_cast<unsigned long long*>(&P.st->total_weight), (unsigned long long)wsum);
+        atomicAdd(reinterpret_cast<unsigned long long*>(&P.st->msf_edges), (unsigned long long)wcnt);
+        atomicAdd(reinterpret_cast<unsigned long long*>(&P.st->winners[g]), (unsigned long long)wcnt);
+    }
+}
+
+// local pass A of shard P.shard: CTA b reads arena b (FIRST: its populate
+// regions), compacts the survivors into the other worklist
+template <bool FIRST>
+__global__ void __launch_bounds__(kBlock, 2) k_dist_passA(Params P, int g, int cur) {
+    __shared__ int s_out;
+    __shared__ long long s_red[3][kWarps];
+    __shared__ int s_pre[kMaxRegionsPerCta + 1];
+    __shared__ int s_rcnt[kMaxRegionsPerCta];
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int b = blockIdx.x;
+    int4* wl[2] = {P.wl0 + (long long)b * P.cap, P.wl1 + (long long)b * P.cap};
+    Src S;
+    if (FIRST) {
+        S.base = nullptr;
+        S.cnt = 0;
+        S.s_pre = s_pre;
+        S.s_rcnt = s_rcnt;
+        S.nreg = b < P.W ? (P.W - b + P.G - 1) / P.G : 0;
+        S.wl0 = P.wl0;
+        S.rcap = P.rcap;
+        S.first_w = b;
+        S.G = P.G;
+        long long canon = 0, heavy = 0;
+        for (int k = tid; k < S.nreg; k += kBlock) {
+            const int4 r = P.region[b + k * P.G];
+            s_rcnt[k] = r.x;
+            canon += r.y;
+            heavy += r.z;
+        }
+        canon = warp_sum(canon);
+        heavy = warp_sum(heavy);
+        if (lane == 0) {
+            s_red[1][warp] = canon;
+            s_red[2][warp] = heavy;
+        }
+        __syncthreads();
+        if (tid == 0) {
+            long long kept = 0;
+            int pre = 0;
+            for (int k = 0; k < S.nreg; ++k) {
+                s_pre[k] = pre;
+                pre += (s_rcnt[k] + kChunk - 1) / kChunk;
+                kept += s_rcnt[k];
+            }
+            s_pre[S.nreg] = pre;
+            canon = heavy = 0;
+            for (int w2 = 0; w2 < kWarps; ++w2) {
+                canon += s_red[1][w2];
+                heavy += s_red[2][w2];
+            }
+            if (kept) atomicAdd(reinterpret_cast<unsigned long long*>(&P.st->live[g - 1]), (unsigned long long)kept);
+            if (g - 1 == 0) {   // phase 1: |E| and the deferred count
+                if (canon) atomicAdd(reinterpret_cast<unsigned long long*>(&P.st->canonical_edges), (unsigned long long)canon);
+                if (heavy) atomicAdd(reinterpret_cast<unsigned long long*>(&P.st->heavy_edges), (unsigned long long)heavy);
+            }
+        }
+        __syncthreads();
+        S.nloc = s_pre[S.nreg];
+    } else {
+        S = compact_src(wl[cur], P.acnt[b]);
+    }
+    if (tid == 0) s_out = 0;
+    __syncthreads();
+    passA(P, S, wl[cur ^ 1], &s_out, P.guards != 0);
+    __syncthreads();
+    if (tid == 0) {
+        P.acnt[b] = s_out;
+        if (s_out) atomicAdd(reinterpret_cast<unsigned long long*>(&P.st->live[g]), (unsigned long long)s_out);
+    }
+}
+
 // ---------------------------------------------------------------------------
 // host side
 // ---------------------------------------------------------------------------
@@ -811,6 +992,7 @@ void ecl_mst_default_options(ecl_mst_options* o) {
     o->max_ctas = 0;
     o->trace = 0;
     o->seed = 0x5eedull;
+    o->threshold_samples = 1024;
 }
 
 size_t ecl_mst_workspace_bytes(int64_t n, int64_t M) {
@@ -893,9 +1075,18 @@ int ecl_mst_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t* n
     P.filter_mode = o.filter < 0 ? -1 : (o.filter ? 1 : 0);
     P.threshold_mode = o.threshold_mode;
     P.threshold_value = o.threshold;
+    P.samples = o.threshold_samples > 0 ? std::min(o.threshold_samples, kMaxSamples) : 20;
     P.halving = o.path_halving ? 1 : 0;
     P.guards = o.atomic_guards < 0 ? -1 : (o.atomic_guards ? 1 : 0);
     P.flatten = o.flatten ? 1 : 0;
+    P.shard = 0;
+    P.nshards = 1;
+    P.nlocal = nchunks;
+    P.zero_mst = 1;
+    P.acnt = nullptr;
+    P.tgt = nullptr;
+    P.keys_all = nullptr;
+    P.nkeys = 1;
     if ((reinterpret_cast<uintptr_t>(nlist) | reinterpret_cast<uintptr_t>(eweight)) % 16 ||
         reinterpret_cast<uintptr_t>(in_mst_out) % 4)
         return fail(ECL_MST_ERR_INVALID, "nlist/eweight must be 16-byte and in_mst 4-byte aligned");
@@ -1086,6 +1277,345 @@ int64_t ecl_mst(int32_t n, const int64_t* nindex, const int32_t* nlist, const in
     }
     if (total == INT64_MIN) fail(ECL_MST_ERR_INPUT, "device found an inconsistent CSR");
     return total;
+}
+
+}  // extern "C"
+
+// ===========================================================================
+// distributed (edge-sharded) path: host side
+// ===========================================================================
+namespace eclmst {
+
+// NCCL is taken from the process at run time (torch's libnccl.so.2 when torch
+// is loaded), so the single-GPU library has no NCCL dependency.
+struct NcclUid {
+    char internal[128];
+};
+typedef void* NcclComm;
+struct NcclApi {
+    bool ok = false;
+    int (*getUniqueId)(NcclUid*) = nullptr;
+    int (*commInitRank)(NcclComm*, int, NcclUid, int) = nullptr;
+    int (*allReduce)(const void*, void*, size_t, int, int, NcclComm, cudaStream_t) = nullptr;
+    int (*commDestroy)(NcclComm) = nullptr;
+    const char* (*getErrorString)(int) = nullptr;
+};
+constexpr int kNcclInt64 = 4, kNcclSum = 0, kNcclMin = 3;
+static NcclApi g_nccl;
+static std::mutex g_nccl_mu;
+
+static int load_nccl() {
+    std::lock_guard<std::mutex> lk(g_nccl_mu);
+    if (g_nccl.ok) return ECL_MST_OK;
+    void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_NOLOAD);
+    const char* env = getenv("ECLMST_NCCL_LIB");
+    if (!h && env) h = dlopen(env, RTLD_NOW);
+    if (!h) h = dlopen("libnccl.so.2", RTLD_NOW);
+    if (!h) return fail(ECL_MST_ERR_CUDA, "libnccl.so.2 not found: %s", dlerror());
+    g_nccl.getUniqueId = reinterpret_cast<int (*)(NcclUid*)>(dlsym(h, "ncclGetUniqueId"));
+    g_nccl.commInitRank = reinterpret_cast<int (*)(NcclComm*, int, NcclUid, int)>(dlsym(h, "ncclCommInitRank"));
+    g_nccl.allReduce = reinterpret_cast<int (*)(const void*, void*, size_t, int, int, NcclComm, cudaStream_t)>(
+        dlsym(h, "ncclAllReduce"));
+    g_nccl.commDestroy = reinterpret_cast<int (*)(NcclComm)>(dlsym(h, "ncclCommDestroy"));
+    g_nccl.getErrorString = reinterpret_cast<const char* (*)(int)>(dlsym(h, "ncclGetErrorString"));
+    if (!g_nccl.getUniqueId || !g_nccl.commInitRank || !g_nccl.allReduce || !g_nccl.commDestroy)
+        return fail(ECL_MST_ERR_CUDA, "libnccl.so.2 lacks the needed symbols");
+    g_nccl.ok = true;
+    return ECL_MST_OK;
+}
+
+struct DistHandle {
+    int rank = 0, world = 1;
+    NcclComm comm = nullptr;
+    long long* h_pin = nullptr;   // pinned host word for the per-round set count
+};
+
+struct DistLayout {
+    size_t stats, internal, rowstart, parent, tgt, keyptrs, shard0, shard_bytes, total;
+    size_t region, acnt, key, wl0, wl1;   // offsets inside one shard block
+    long long wl_cap, nlocal_max;
+};
+
+static inline DistLayout dist_layout(int64_t n, int64_t M, int S, int world) {
+    DistLayout L;
+    const long long nchunks = ceil_div(M, kChunk);
+    const long long P = (long long)S * world;
+    L.nlocal_max = ceil_div(nchunks, P);
+    const long long wmax = L.nlocal_max < kMaxPopWarps ? L.nlocal_max : kMaxPopWarps;
+    L.wl_cap = (L.nlocal_max + wmax) * kChunk;
+    size_t off = 0;
+    L.stats = off;    off = align_up(off + sizeof(ecl_mst_stats), 256);
+    L.internal = off; off = align_up(off + sizeof(Internal), 256);
+    L.rowstart = off; off = align_up(off + sizeof(int) * (size_t)(nchunks + 1), 256);
+    L.parent = off;   off = align_up(off + sizeof(int) * (size_t)n, 256);
+    L.tgt = off;      off = align_up(off + sizeof(int) * (size_t)n, 256);
+    L.keyptrs = off;  off = align_up(off + sizeof(long long*) * (size_t)S, 256);
+    size_t so = 0;
+    L.region = so; so = align_up(so + sizeof(int4) * (size_t)kMaxPopWarps, 256);
+    L.acnt = so;   so = align_up(so + sizeof(int) * (size_t)kMaxGrid, 256);
+    L.key = so;    so = align_up(so + sizeof(long long) * (size_t)n, 256);
+    L.wl0 = so;    so = align_up(so + sizeof(int4) * (size_t)L.wl_cap, 256);
+    L.wl1 = so;    so = align_up(so + sizeof(int4) * (size_t)L.wl_cap, 256);
+    L.shard_bytes = so;
+    L.shard0 = off;
+    off += so * (size_t)S;
+    L.total = off;
+    return L;
+}
+
+}  // namespace eclmst
+
+extern "C" {
+
+int ecl_mst_dist_unique_id(void* uid_out) {
+    g_last_error.clear();
+    if (!uid_out) return fail(ECL_MST_ERR_INVALID, "null argument");
+    int rc = load_nccl();
+    if (rc) return rc;
+    int r = g_nccl.getUniqueId(reinterpret_cast<NcclUid*>(uid_out));
+    if (r) return fail(ECL_MST_ERR_CUDA, "ncclGetUniqueId: %d", r);
+    return ECL_MST_OK;
+}
+
+int ecl_mst_dist_init(const void* uid, int32_t rank, int32_t world, void** handle_out) {
+    g_last_error.clear();
+    if (!handle_out || world < 1 || rank < 0 || rank >= world) return fail(ECL_MST_ERR_INVALID, "bad rank/world");
+    DistHandle* h = new DistHandle;
+    h->rank = rank;
+    h->world = world;
+    cudaError_t e = cudaHostAlloc(reinterpret_cast<void**>(&h->h_pin), sizeof(long long) * 4, cudaHostAllocDefault);
+    if (e != cudaSuccess) {
+        delete h;
+        return fail(ECL_MST_ERR_CUDA, "cudaHostAlloc: %s", cudaGetErrorString(e));
+    }
+    if (world > 1 || uid) {   // world 1 with a uid: a one-rank NCCL communicator (tests the NCCL path)
+        if (!uid) {
+            cudaFreeHost(h->h_pin);
+            delete h;
+            return fail(ECL_MST_ERR_INVALID, "world > 1 needs an NCCL unique id");
+        }
+        int rc = load_nccl();
+        NcclUid id;
+        if (!rc) {
+            std::memcpy(id.internal, uid, sizeof id.internal);
+            const int r = g_nccl.commInitRank(&h->comm, world, id, rank);
+            if (r) rc = fail(ECL_MST_ERR_CUDA, "ncclCommInitRank: %s", g_nccl.getErrorString ? g_nccl.getErrorString(r) : "?");
+        }
+        if (rc) {
+            cudaFreeHost(h->h_pin);
+            delete h;
+            return rc;
+        }
+    }
+    *handle_out = h;
+    return ECL_MST_OK;
+}
+
+int ecl_mst_dist_finalize(void* handle) {
+    g_last_error.clear();
+    DistHandle* h = static_cast<DistHandle*>(handle);
+    if (!h) return ECL_MST_OK;
+    if (h->comm && g_nccl.ok) g_nccl.commDestroy(h->comm);
+    if (h->h_pin) cudaFreeHost(h->h_pin);
+    delete h;
+    return ECL_MST_OK;
+}
+
+int64_t ecl_mst_dist_shard_chunks(int64_t M, int32_t shard, int32_t nshards) {
+    if (M < 0 || nshards < 1 || shard < 0 || shard >= nshards) return -1;
+    const long long nchunks = ceil_div(M, kChunk);
+    return shard < nchunks ? (nchunks - shard + nshards - 1) / nshards : 0;
+}
+
+size_t ecl_mst_dist_workspace_bytes(int64_t n, int64_t M, int32_t local_shards, int32_t world) {
+    if (n < 0 || n > INT32_MAX || M < 0 || M > (int64_t)0xFFFFFFFFLL || local_shards < 1 || world < 1) return 0;
+    return dist_layout(n, M, local_shards, world).total;
+}
+
+int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M, const int64_t* nindex,
+                        const int32_t* nlist, const int32_t* eweight, uint8_t* in_mst_out,
+                        int64_t* total_weight_out, void* workspace, size_t workspace_bytes,
+                        const ecl_mst_options* opts, void* stream) {
+    g_last_error.clear();
+    DistHandle* h = static_cast<DistHandle*>(handle);
+    if (!h) return fail(ECL_MST_ERR_INVALID, "null handle (ecl_mst_dist_init)");
+    const int S = local_shards, world = h->world, rank = h->rank;
+    if (S < 1 || S > 64) return fail(ECL_MST_ERR_INVALID, "local_shards must be in [1, 64]");
+    if (world > 1 && S != 1) return fail(ECL_MST_ERR_INVALID, "local_shards > 1 only without NCCL (world 1)");
+    if (n < 0 || M < 0) return fail(ECL_MST_ERR_INVALID, "negative n or M");
+    if (M > (int64_t)0xFFFFFFFFLL) return fail(ECL_MST_ERR_TOO_LARGE, "M exceeds 2^32-1");
+    if (!total_weight_out || !workspace || (n > 0 && !nindex) || (M > 0 && (!nlist || !eweight || !in_mst_out)))
+        return fail(ECL_MST_ERR_INVALID, "null argument");
+    if (M > 0 && n == 0) return fail(ECL_MST_ERR_INVALID, "M > 0 with n = 0");
+    const DistLayout L = dist_layout(n, M, S, world);
+    if (workspace_bytes < L.total) return fail(ECL_MST_ERR_WORKSPACE, "workspace %zu < %zu bytes", workspace_bytes, L.total);
+    if (reinterpret_cast<uintptr_t>(workspace) % 256) return fail(ECL_MST_ERR_WORKSPACE, "workspace not 256-byte aligned");
+    if ((reinterpret_cast<uintptr_t>(nlist) | reinterpret_cast<uintptr_t>(eweight)) % 16 ||
+        reinterpret_cast<uintptr_t>(in_mst_out) % 4)
+        return fail(ECL_MST_ERR_INVALID, "nlist/eweight must be 16-byte and in_mst 4-byte aligned");
+    ecl_mst_options o;
+    ecl_mst_default_options(&o);
+    if (opts) o = *opts;
+    cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
+    char* ws = static_cast<char*>(workspace);
+    ecl_mst_stats* st = reinterpret_cast<ecl_mst_stats*>(ws + L.stats);
+    Internal* in = reinterpret_cast<Internal*>(ws + L.internal);
+    if (M == 0) {
+        cudaError_t e = cudaMemsetAsync(st, 0, sizeof(ecl_mst_stats), s);
+        if (e == cudaSuccess) e = cudaMemsetAsync(total_weight_out, 0, sizeof(int64_t), s);
+        if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "memset: %s", cudaGetErrorString(e));
+        return ECL_MST_OK;
+    }
+    DevInfo di;
+    int rc = device_info(&di);
+    if (rc) return rc;
+    const long long nchunks = ceil_div(M, kChunk);
+    const long long Pt = (long long)S * world;
+
+    // per-shard launch geometry and parameters
+    std::vector<Params> sp(S);
+    std::vector<long long*> keyptr(S);
+    for (int k = 0; k < S; ++k) keyptr[k] = reinterpret_cast<long long*>(ws + L.shard0 + k * L.shard_bytes + L.key);
+    long long** d_keyptrs = reinterpret_cast<long long**>(ws + L.keyptrs);
+    cudaError_t e = cudaMemcpyAsync(d_keyptrs, keyptr.data(), sizeof(long long*) * S, cudaMemcpyHostToDevice, s);
+    for (int k = 0; k < S; ++k) {
+        Params& P = sp[k];
+        std::memset(&P, 0, sizeof P);
+        const int shard = rank * S + k;
+        const long long nlocal = shard < nchunks ? (nchunks - shard + Pt - 1) / Pt : 0;
+        long long G = (long long)di.sms * di.occ;
+        if (G > std::max<long long>(nlocal, 1)) G = std::max<long long>(nlocal, 1);
+        if (G > kMaxGrid) G = kMaxGrid;
+        long long W = (long long)di.sms * di.pop_occ * kPopWarps;
+        if (W > std::max<long long>(nlocal, 1)) W = std::max<long long>(nlocal, 1);
+        if (W > kMaxPopWarps) W = kMaxPopWarps;
+        if (W > G * kMaxRegionsPerCta) W = G * kMaxRegionsPerCta;
+        W = std::max<long long>(1, W / G) * G;
+        const long long rcap = std::max<long long>(1, ceil_div(nlocal, W)) * kChunk;
+        const long long cap = (W / G) * rcap;
+        if (W * rcap > L.wl_cap || cap >= (1LL << 30)) return fail(ECL_MST_ERR_TOO_LARGE, "shard worklist too large");
+        char* sb = ws + L.shard0 + k * L.shard_bytes;
+        P.n = n;
+        P.M = M;
+        P.nchunks = nchunks;
+        P.G = (int)G;
+        P.cap = cap;
+        P.W = (int)W;
+        P.rcap = rcap;
+        P.nindex = reinterpret_cast<const long long*>(nindex);
+        P.nlist = nlist;
+        P.eweight = eweight;
+        P.in_mst = in_mst_out;
+        P.total_out = reinterpret_cast<long long*>(total_weight_out);
+        P.st = st;
+        P.in = in;
+        P.trace = nullptr;
+        P.rowstart = reinterpret_cast<int*>(ws + L.rowstart);
+        P.region = reinterpret_cast<int4*>(sb + L.region);
+        P.key = keyptr[k];
+        P.parent = reinterpret_cast<int*>(ws + L.parent);
+        P.wl0 = reinterpret_cast<int4*>(sb + L.wl0);
+        P.wl1 = reinterpret_cast<int4*>(sb + L.wl1);
+        P.seed = o.seed;
+        P.filter_mode = o.filter < 0 ? -1 : (o.filter ? 1 : 0);
+        P.threshold_mode = o.threshold_mode;
+        P.threshold_value = o.threshold;
+        P.samples = o.threshold_samples > 0 ? std::min(o.threshold_samples, kMaxSamples) : 20;
+        P.halving = o.path_halving ? 1 : 0;
+        P.guards = o.atomic_guards == 0 ? 0 : 1;
+        P.flatten = o.flatten ? 1 : 0;
+        P.shard = shard;
+        P.nshards = (int)Pt;
+        P.nlocal = nlocal;
+        P.zero_mst = 0;
+        P.acnt = reinterpret_cast<int*>(sb + L.acnt);
+        P.tgt = reinterpret_cast<int*>(ws + L.tgt);
+        P.keys_all = d_keyptrs;
+        P.nkeys = S;
+    }
+    Params& P0 = sp[0];
+    const unsigned vblocks = (unsigned)std::max<long long>(1, std::min<long long>(ceil_div((long long)n, 256), (long long)di.sms * 8));
+    auto check = [&](const char* what) -> int {
+        cudaError_t e2 = cudaGetLastError();
+        if (e2 != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "%s: %s", what, cudaGetErrorString(e2));
+        return ECL_MST_OK;
+    };
+    auto allreduce = [&](void* buf, size_t count, int op) -> int {
+        if (!h->comm) return ECL_MST_OK;
+        const int r = g_nccl.allReduce(buf, buf, count, kNcclInt64, op, h->comm, s);
+        if (r) return fail(ECL_MST_ERR_CUDA, "ncclAllReduce: %s", g_nccl.getErrorString ? g_nccl.getErrorString(r) : "?");
+        return ECL_MST_OK;
+    };
+    auto read_word = [&](const void* dptr, long long* out) -> int {
+        cudaError_t e2 = cudaMemcpyAsync(h->h_pin, dptr, sizeof(long long), cudaMemcpyDeviceToHost, s);
+        if (e2 == cudaSuccess) e2 = cudaStreamSynchronize(s);
+        if (e2 != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "sync: %s", cudaGetErrorString(e2));
+        *out = *h->h_pin;
+        return ECL_MST_OK;
+    };
+
+    if (e == cudaSuccess) e = cudaMemsetAsync(st, 0, sizeof(ecl_mst_stats), s);
+    if (e == cudaSuccess) e = cudaMemsetAsync(in_mst_out, 0, (size_t)M, s);   // every rank returns the full mask
+    if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "memset: %s", cudaGetErrorString(e));
+    k_init<<<vblocks, 256, 0, s>>>(P0);
+    if ((rc = check("k_init"))) return rc;
+    int g = 0;
+    for (int ph = 1; ph <= 2; ++ph) {
+        if (ph == 2) {
+            // the phase-2 decision needs the global deferred count
+            if ((rc = allreduce(&st->canonical_edges, 2, kNcclSum))) return rc;
+            long long filtered = 0, heavy = 0;
+            if ((rc = read_word(&st->heavy_edges, &heavy))) return rc;
+            if ((rc = read_word(&st->filtered, &filtered))) return rc;
+            if (!(filtered & 0xffffffffll) || heavy == 0) break;
+            k_flatten<1><<<vblocks, 256, 0, s>>>(P0);
+            k_flatten<2><<<vblocks, 256, 0, s>>>(P0);
+            ++g;
+            if (g >= ECL_MST_MAX_ROUNDS) return fail(ECL_MST_ERR_INPUT, "round limit");
+            e = cudaMemcpyAsync(&st->phase2_round, &g, sizeof(int), cudaMemcpyHostToDevice, s);
+            if (e == cudaSuccess) e = cudaStreamSynchronize(s);   // &g is a host stack value
+            if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "phase2: %s", cudaGetErrorString(e));
+        }
+        for (int k = 0; k < S; ++k) {
+            if (ph == 1) k_populate<1><<<(unsigned)ceil_div(sp[k].W, kPopWarps), kPopBlock, 0, s>>>(sp[k]);
+            else k_populate<2><<<(unsigned)ceil_div(sp[k].W, kPopWarps), kPopBlock, 0, s>>>(sp[k]);
+        }
+        if ((rc = check("populate"))) return rc;
+        bool first = true;
+        int cur = 0;
+        while (true) {
+            // allreduce(min) of the best-edge keys over all shards
+            if (S > 1) k_vreduce<<<vblocks, 256, 0, s>>>(P0);
+            if ((rc = allreduce(P0.key, (size_t)n, kNcclMin))) return rc;
+            e = cudaMemsetAsync(&in->reps, 0, sizeof(in->reps), s);
+            if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "memset: %s", cudaGetErrorString(e));
+            k_dist_reps1<<<vblocks, 256, 0, s>>>(P0);
+            long long reps = 0;
+            if ((rc = read_word(&in->reps, &reps))) return rc;
+            if (reps == 0) {
+                if (first)
+                    for (int k = 0; k < S; ++k) k_dist_passA<true><<<sp[k].G, kBlock, 0, s>>>(sp[k], g + 1, cur);
+                break;   // no set has a live edge anywhere: the phase is done
+            }
+            k_dist_reps2<<<vblocks, 256, 0, s>>>(P0, g);
+            if (g + 1 >= ECL_MST_MAX_ROUNDS) return fail(ECL_MST_ERR_INPUT, "round limit");
+            ++g;
+            for (int k = 0; k < S; ++k) {
+                if (first) k_dist_passA<true><<<sp[k].G, kBlock, 0, s>>>(sp[k], g, cur);
+                else k_dist_passA<false><<<sp[k].G, kBlock, 0, s>>>(sp[k], g, cur);
+            }
+            cur ^= 1;
+            first = false;
+            if ((rc = check("rounds"))) return rc;
+        }
+    }
+    const int rounds = g + 1;
+    e = cudaMemcpyAsync(&st->rounds, &rounds, sizeof(int), cudaMemcpyHostToDevice, s);
+    if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "stats: %s", cudaGetErrorString(e));
+    k_finalize<<<1, 32, 0, s>>>(P0);
+    if ((rc = check("finalize"))) return rc;
+    return ECL_MST_OK;
 }
 
 }  // extern "C"

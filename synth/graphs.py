@@ -103,51 +103,69 @@ def csr_from_pairs(n: int, u: torch.Tensor, v: torch.Tensor, wfn, name: str = ""
     come from wfn(a, b) with a < b, so both directions agree and the builder
     never has to carry weights through the sort.
     """
-    dev = u.device
     u = u.to(torch.int64)
     v = v.to(torch.int64)
     keep = u != v
     u, v = u[keep], v[keep]
-    a = torch.minimum(u, v)
-    b = torch.maximum(u, v)
+    keys = torch.minimum(u, v) * n + torch.maximum(u, v)
     del u, v, keep
-    canon = torch.unique(a * n + b)          # sorted, deduplicated canonical pairs
-    del a, b
-    m = canon.numel()
-    a = canon // n
-    b = canon - a * n
-    del canon
-    keys = torch.cat([a * n + b, b * n + a])
-    del a, b
-    keys = torch.sort(keys).values if keys.numel() <= (1 << 31) - 1 else _chunked_sort(keys)
-    src = keys // n
-    dst = keys - src * n
+    return csr_from_keys(n, keys, wfn, name, chunk)
+
+
+def csr_from_keys(n: int, keys: torch.Tensor, wfn, name: str = "", chunk: int = 1 << 28) -> Graph:
+    """As csr_from_pairs, from canonical keys a*n + b (a < b, duplicates allowed).
+    Works in chunks so a 1e9-edge graph fits comfortably in one GPU."""
+    dev = keys.device
+    canon = torch.unique(keys)          # sorted, deduplicated canonical pairs
     del keys
-    counts = torch.bincount(src, minlength=n)
+    m = canon.numel()
+    mirror = torch.empty_like(canon)
+    for s in range(0, m, chunk):
+        a = canon[s:s + chunk] // n
+        mirror[s:s + chunk] = (canon[s:s + chunk] - a * n) * n + a
+    allk = _sorted_union(canon, mirror)  # both directions, sorted by (src, dst)
+    del canon, mirror
+    M = allk.numel()
+    counts = torch.zeros(n, dtype=torch.int64, device=dev)
+    nlist = torch.empty(M, dtype=torch.int32, device=dev)
+    eweight = torch.empty(M, dtype=torch.int32, device=dev)
+    for s in range(0, M, chunk):
+        k = allk[s:s + chunk]
+        src = k // n
+        dst = k - src * n
+        counts += torch.bincount(src, minlength=n)
+        nlist[s:s + chunk] = dst.to(torch.int32)
+        eweight[s:s + chunk] = wfn(torch.minimum(src, dst), torch.maximum(src, dst)).to(torch.int32)
+        del k, src, dst
+    del allk
     nindex = torch.zeros(n + 1, dtype=torch.int64, device=dev)
     nindex[1:] = torch.cumsum(counts, 0)
-    del counts
-    eweight = torch.empty(src.numel(), dtype=torch.int32, device=dev)
-    for s in range(0, src.numel(), chunk):
-        x, y = src[s:s + chunk], dst[s:s + chunk]
-        eweight[s:s + chunk] = wfn(torch.minimum(x, y), torch.maximum(x, y)).to(torch.int32)
-    del src
-    g = Graph(n, nindex, dst.to(torch.int32), eweight, name)
+    g = Graph(n, nindex, nlist, eweight, name)
     g.meta["m_undirected"] = int(m)
     return g
 
 
-def _chunked_sort(keys: torch.Tensor) -> torch.Tensor:  # pragma: no cover - huge inputs only
-    lo = int(keys.min())
-    hi = int(keys.max()) + 1
-    parts = []
-    nb = 4
-    step = (hi - lo + nb - 1) // nb
-    for i in range(nb):
-        sel = keys[(keys >= lo + i * step) & (keys < lo + (i + 1) * step)]
-        parts.append(torch.sort(sel).values)
-        del sel
-    return torch.cat(parts)
+def _sorted_union(a: torch.Tensor, b: torch.Tensor, buckets: int = 8) -> torch.Tensor:
+    """Sorted concatenation of two disjoint sorted int64 tensors (key-range
+    buckets keep every individual sort well below 2^31 elements)."""
+    total = a.numel() + b.numel()
+    if total <= (1 << 29):
+        return torch.sort(torch.cat([a, b])).values
+    lo = min(int(a[0]), int(b.min()))
+    hi = max(int(a[-1]), int(b.max())) + 1
+    step = (hi - lo + buckets - 1) // buckets
+    out = torch.empty(total, dtype=a.dtype, device=a.device)
+    pos = 0
+    for i in range(buckets):
+        x0, x1 = lo + i * step, lo + (i + 1) * step
+        ia0, ia1 = torch.searchsorted(a, torch.tensor([x0, x1], device=a.device)).tolist()
+        part_b = b[(b >= x0) & (b < x1)]
+        part = torch.sort(torch.cat([a[ia0:ia1], part_b])).values
+        out[pos:pos + part.numel()] = part
+        pos += part.numel()
+        del part, part_b
+    assert pos == total
+    return out
 
 
 def _hash_weight(seed: int, n: int):
@@ -288,7 +306,8 @@ def rmat(scale: int = 24, edge_factor: int = 16, a: float = 0.57, b: float = 0.1
     tA = int(a * (1 << 53))
     tAB = int((a + b) * (1 << 53))
     tABC = int((a + b + c) * (1 << 53))
-    us, vs = [], []
+    perm = _random_permutation(n, seed, device)
+    parts = []
     for s0 in range(0, m_draws, chunk):
         d = torch.arange(s0, min(m_draws, s0 + chunk), dtype=torch.int64, device=device)
         u = torch.zeros_like(d)
@@ -299,16 +318,16 @@ def rmat(scale: int = 24, edge_factor: int = 16, a: float = 0.57, b: float = 0.1
             vb = (((r >= tA) & (r < tAB)) | (r >= tABC)).to(torch.int64)
             u = u | (ub << (scale - 1 - lvl))
             v = v | (vb << (scale - 1 - lvl))
-        us.append(u)
-        vs.append(v)
-    u = torch.cat(us)
-    v = torch.cat(vs)
-    del us, vs
-    perm = _random_permutation(n, seed, device)
-    u = perm[u]
-    v = perm[v]
+        u = perm[u]
+        v = perm[v]
+        keep = u != v
+        u, v = u[keep], v[keep]
+        parts.append(torch.minimum(u, v) * n + torch.maximum(u, v))
+        del d, u, v, keep
     del perm
-    g = csr_from_pairs(n, u, v, _hash_weight(seed, n), name=f"rmat{scale}")
+    keys = torch.cat(parts)
+    del parts
+    g = csr_from_keys(n, keys, _hash_weight(seed, n), name=f"rmat{scale}")
     g.meta.update(family="rmat", seed=seed, scale=scale, edge_factor=edge_factor)
     return g
 
@@ -316,15 +335,18 @@ def rmat(scale: int = 24, edge_factor: int = 16, a: float = 0.57, b: float = 0.1
 def uniform_random(n: int = 1 << 26, m_draws: int = 1_000_000_000, seed: int = 5,
                    device="cpu", chunk: int = 1 << 27) -> Graph:
     """C5: uniform random graph G(n, m) (Table 2 'r4-2e23.sym')."""
-    us, vs = [], []
+    parts = []
     for s0 in range(0, m_draws, chunk):
         d = torch.arange(s0, min(m_draws, s0 + chunk), dtype=torch.int64, device=device)
-        us.append(rng.below(seed, _S_U, d, n))
-        vs.append(rng.below(seed, _S_V, d, n))
-    u = torch.cat(us)
-    v = torch.cat(vs)
-    del us, vs
-    g = csr_from_pairs(n, u, v, _hash_weight(seed, n), name=f"uniform{n}")
+        u = rng.below(seed, _S_U, d, n)
+        v = rng.below(seed, _S_V, d, n)
+        keep = u != v
+        u, v = u[keep], v[keep]
+        parts.append(torch.minimum(u, v) * n + torch.maximum(u, v))
+        del d, u, v, keep
+    keys = torch.cat(parts)
+    del parts
+    g = csr_from_keys(n, keys, _hash_weight(seed, n), name=f"uniform{n}")
     g.meta.update(family="uniform", seed=seed, m_draws=m_draws)
     return g
 

@@ -93,6 +93,7 @@ def test_config_small(eclmst, name):
     dict(filter=1, threshold_mode=1, threshold=(1 << 31) - 1), dict(filter=1, threshold_mode=1, threshold=0),
     dict(seed=1), dict(seed=12345), dict(path_halving=0), dict(max_ctas=1), dict(max_ctas=7),
     dict(atomic_guards=0), dict(atomic_guards=1), dict(flatten=0), dict(flatten=0, path_halving=0), dict(trace=1),
+    dict(threshold_samples=20), dict(threshold_samples=4096, seed=7),
 ])
 @pytest.mark.parametrize("name", ["rmat", "uniform", "road"])
 def test_knobs_give_identical_msf(eclmst, name, opts):
