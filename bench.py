@@ -51,6 +51,7 @@ def parse():
     ap.add_argument("--no-parity", action="store_true")
     ap.add_argument("--flush-mb", type=int, default=512)
     ap.add_argument("--opt", action="append", default=[], help="ecl_mst_options field=value (ablations)")
+    ap.add_argument("--dist", action="store_true", help="use the edge-sharded NCCL path even on one GPU")
     return ap.parse_args()
 
 
@@ -239,7 +240,7 @@ def run_reference(args, rank, world):
     line = {
         "impl": "reference", "metric": METRIC, "value": value, "unit": "edges/s", "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
-        "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+        "scaling": "strong", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
         "config": {"workload": f"{CONFIG_NAMES[args.config]} {g.name}", "n": g.n, "M": g.M},
         "cpu_baseline": {"value": value, "unit": "edges/s", "cores": 1, "kind": "oracle",
                          "sample": f"whole {g.name} graph per step (serial C Kruskal, oracle/kruskal.c)"},
@@ -259,9 +260,17 @@ def main():
 
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
+    use_dist = world > 1 or args.dist
     if world > 1:
         import torch.distributed as dist
         dist.init_process_group("nccl", device_id=dev)
+    elif use_dist:
+        import socket
+        import torch.distributed as dist
+        with socket.socket() as sk:
+            sk.bind(("127.0.0.1", 0))
+            port = sk.getsockname()[1]
+        dist.init_process_group("nccl", init_method=f"tcp://127.0.0.1:{port}", rank=0, world_size=1, device_id=dev)
     eclmst.load()   # fails loudly if libeclmst.so is missing
 
     t_gen = time.perf_counter()
@@ -270,7 +279,12 @@ def main():
     t_gen = time.perf_counter() - t_gen
     n, M = g.n, g.M
 
-    ws_bytes = eclmst.ecl_mst_workspace_bytes(n, M)
+    handle = None
+    if use_dist:   # edge-sharded path: NCCL allreduce(min) per round inside the library
+        handle = eclmst.dist.init_from_group()
+        ws_bytes = eclmst.ecl_mst_dist_workspace_bytes(n, M, 1, world)
+    else:
+        ws_bytes = eclmst.ecl_mst_workspace_bytes(n, M)
     ws = torch.empty(ws_bytes, dtype=torch.uint8, device=dev)
     in_mst = torch.empty(M, dtype=torch.uint8, device=dev)
     total = torch.empty(1, dtype=torch.int64, device=dev)
@@ -278,11 +292,17 @@ def main():
     stream = torch.cuda.current_stream()
     opt_kw = {k: int(v) for k, v in (o.split("=", 1) for o in args.opt)}
     opts = eclmst.default_options(**opt_kw)
-    opts.trace |= 2     # CUDA events between the library's kernels (per-kernel roofline)
+    if not use_dist:
+        opts.trace |= 2     # CUDA events between the library's kernels (per-kernel roofline)
 
     def step():
-        eclmst.ecl_mst_device(n, g.nindex, g.nlist, g.eweight, in_mst_out=in_mst, total_weight_out=total,
-                              workspace=ws, options=opts, stream=stream)
+        if not use_dist:
+            eclmst.ecl_mst_device(n, g.nindex, g.nlist, g.eweight, in_mst_out=in_mst, total_weight_out=total,
+                                  workspace=ws, options=opts, stream=stream)
+        else:
+            eclmst.ecl_mst_dist_device(handle, n, g.nindex, g.nlist, g.eweight, local_shards=1, world=world,
+                                       in_mst_out=in_mst, total_weight_out=total, workspace=ws, options=opts,
+                                       stream=stream)
 
     for _ in range(max(args.warmup, 3)):
         flush.zero_()
@@ -292,7 +312,7 @@ def main():
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
     sampler = ClockSampler(local)
     sampler.start()
-    if world > 1:
+    if use_dist:
         torch.distributed.barrier()
     torch.cuda.synchronize()
     wall0 = time.perf_counter()
@@ -302,16 +322,17 @@ def main():
         ev[i][0].record(stream)
         step()
         ev[i][1].record(stream)
-        kern.append(eclmst.ecl_mst_kernel_times())   # waits for this step's events
+        if not use_dist:
+            kern.append(eclmst.ecl_mst_kernel_times())   # waits for this step's events
     torch.cuda.synchronize()
-    if world > 1:
+    if use_dist:
         torch.distributed.barrier()
     wall = time.perf_counter() - wall0
     clocks = sampler.stop()
     per_step = [a.elapsed_time(b) for a, b in ev]
     ms = sum(per_step) / len(per_step)
     ms_max = ms
-    if world > 1:
+    if use_dist:
         t = torch.tensor([ms], device=dev)
         torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
         ms_max = float(t.item())
@@ -321,7 +342,38 @@ def main():
 
     # ---- e2e through the host C-ABI call (pinned host buffers, copies timed) ----
     e2e = None
-    if not args.no_e2e:
+    if not args.no_e2e and use_dist:
+        # sharded e2e through the public API: pinned host CSR -> device, run, mask -> host
+        h_idx = g.nindex.cpu().pin_memory()
+        h_list = g.nlist.cpu().pin_memory()
+        h_w = g.eweight.cpu().pin_memory()
+        h_out = torch.empty(M, dtype=torch.uint8).pin_memory()
+        d_idx = torch.empty_like(g.nindex)
+        d_list = torch.empty_like(g.nlist)
+        d_w = torch.empty_like(g.eweight)
+        et = []
+        for i in range(args.steps + 1):
+            torch.distributed.barrier()
+            t0 = time.perf_counter()
+            d_idx.copy_(h_idx, non_blocking=True)
+            d_list.copy_(h_list, non_blocking=True)
+            d_w.copy_(h_w, non_blocking=True)
+            eclmst.ecl_mst_dist_device(handle, n, d_idx, d_list, d_w, local_shards=1, world=world,
+                                       in_mst_out=in_mst, total_weight_out=total, workspace=ws, options=opts,
+                                       stream=stream)
+            h_out.copy_(in_mst, non_blocking=True)
+            tot_h = int(total.item())
+            if i:
+                et.append(time.perf_counter() - t0)
+        e_ms = 1e3 * sum(et) / len(et)
+        t = torch.tensor([e_ms], device=dev)
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+        e_ms = float(t.item())
+        e2e = {"value": M / (e_ms / 1e3), "unit": "edges/s",
+               "h2d_bytes_per_step": 8 * (n + 1) + 8 * M, "d2h_bytes_per_step": M + 8,
+               "ms_per_step": e_ms, "same_result": tot_h == result_total,
+               "path": "ecl_mst_dist_device with pinned host->device copies (every rank holds the CSR)"}
+    if not args.no_e2e and not use_dist:
         h_idx = g.nindex.cpu().pin_memory()
         h_list = g.nlist.cpu().pin_memory()
         h_w = g.eweight.cpu().pin_memory()
@@ -335,16 +387,13 @@ def main():
             et.append(time.perf_counter() - t0)
         eclmst.ecl_mst_release_host_cache()
         e_ms = 1e3 * sum(et) / len(et)
-        if world > 1:
-            t = torch.tensor([e_ms], device=dev)
-            torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
-            e_ms = float(t.item())
-        e2e = {"value": world * M / (e_ms / 1e3), "unit": "edges/s",
+        e2e = {"value": M / (e_ms / 1e3), "unit": "edges/s",
                "h2d_bytes_per_step": 8 * (n + 1) + 8 * M, "d2h_bytes_per_step": M + 8,
                "ms_per_step": e_ms, "same_result": tot_h == result_total}
 
     if rank != 0:
-        if world > 1:
+        if use_dist:
+            eclmst.ecl_mst_dist_finalize(handle)
             torch.distributed.destroy_process_group()
         return
 
@@ -380,31 +429,38 @@ def main():
 
     peak, peak_src = load_peaks()
     ab = algorithmic_bytes(n, M, st)
-    kern_ms = {k: sum(d[k] for d in kern) / len(kern) for k in kern[0]}
-    dominant = max(("populate1", "rounds1", "populate2", "rounds2", "init", "flatten"), key=lambda k: kern_ms[k])
-    achieved = ab[dominant] / (kern_ms[dominant] / 1e3) / 1e9
+    if kern:
+        kern_ms = {k: sum(d[k] for d in kern) / len(kern) for k in kern[0]}
+        dominant = max(("populate1", "rounds1", "populate2", "rounds2", "init", "flatten"), key=lambda k: kern_ms[k])
+    else:   # sharded run: no per-kernel events; the whole step is the unit
+        kern_ms = {"total": ms_max}
+        ab["total_step"] = ab["total"]
+        dominant = "total_step"
+    achieved = ab[dominant] / (kern_ms.get(dominant, ms_max) / 1e3) / 1e9
     prof = load_traffic()
     traffic = None
     if prof and prof.get("workload") == g.name:
         traffic = prof.get("dram_bytes_per_launch", {}).get(dominant)
-    value = world * M / (ms_max / 1e3)
+    value = M / (ms_max / 1e3)   # one graph per step, whatever N (strong scaling)
     line = {
         "metric": METRIC, "value": value, "unit": "edges/s", "n_gpus": world, "steps": args.steps,
         "warmup": max(args.warmup, 3), "ms_per_step": ms_max, "higher_is_better": True,
-        "scaling": "weak", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+        "scaling": "strong", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
         "config": {"workload": f"{CONFIG_NAMES[args.config]} {g.name}", "n": n, "M": M,
-                   "m_undirected": st["canonical_edges"], "parallelism": "replicas" if world > 1 else "single",
+                   "m_undirected": st["canonical_edges"],
+                   "parallelism": (f"edge-sharded x{world} (ncclAllReduce min per round, replicated union-find)"
+                                   if use_dist else "single GPU"),
                    "options": opt_kw,
                    "l2": f"inputs ({(8 * M + 8 * n) / 1e6:.0f} MB CSR) exceed L2; plus {args.flush_mb} MB flush "
                          "between steps"},
         "ms_per_graph": ms_max, "ms_per_step_all": per_step, "wall_s": wall,
-        "edges_per_s_undirected": world * st["canonical_edges"] / (ms_max / 1e3),
-        "gpu_launches": args.steps * LAUNCHES_PER_STEP,
+        "edges_per_s_undirected": st["canonical_edges"] / (ms_max / 1e3),
+        "gpu_launches": args.steps * (LAUNCHES_PER_STEP if not use_dist else 4 + 4 * st["rounds"]),
         "clocks": clocks,
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
-                     "kernel": KERNEL_OF_STAGE[dominant], "stage": dominant,
-                     "kernel_share_of_step": kern_ms[dominant] / ms,
+                     "kernel": KERNEL_OF_STAGE.get(dominant, "all (sharded step)"), "stage": dominant,
+                     "kernel_share_of_step": kern_ms.get(dominant, ms_max) / ms,
                      "algorithmic_bytes_per_launch": ab[dominant],
                      "whole_step": {"algorithmic_bytes": ab["total"],
                                     "achieved_gbs": ab["total"] / (ms / 1e3) / 1e9,
@@ -415,11 +471,13 @@ def main():
         "parity_vs_oracle": parity,
         "stats": {"rounds": st["rounds"], "filtered": st["filtered"], "threshold": st["threshold"],
                   "phase2_round": st["phase2_round"], "grid": st["grid"], "msf_edges": st["msf_edges"],
-                  "live": st["live"], "winners": st["winners"], "stage_us": stage_times(st)},
+                  "live": st["live"], "winners": st["winners"],
+                  "stage_us": None if use_dist else stage_times(st)},
         "gen_s": t_gen,
     }
     print(json.dumps(line), flush=True)
-    if world > 1:
+    if use_dist:
+        eclmst.ecl_mst_dist_finalize(handle)
         torch.distributed.destroy_process_group()
 
 
