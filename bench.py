@@ -30,7 +30,9 @@ import torch  # noqa: E402
 
 PEAKS_FILE = os.path.join(ROOT, "MEASURED_PEAKS.json")
 PROFILE_SUMMARY = os.path.join(ROOT, "profiles", "ncu_summary_latest.json")
-LAUNCHES_PER_STEP = 8   # k_init, k_populate<1>, k_rounds<1>, k_flatten<1>, k_flatten<2>, k_populate<2>, k_rounds<2>, k_finalize
+# k_init, k_populate<1>, k_rounds<1>, k_finalize; with filtering also k_flatten<1>, k_flatten<2>,
+# k_populate<2>, k_rounds<2>
+LAUNCHES_UNFILTERED, LAUNCHES_FILTERED = 4, 8
 CONFIG_NAMES = {"grid": "C1", "road": "C2", "rgg": "C3", "rmat": "C4", "uniform": "C5"}
 METRIC = "MSF edges/sec and ms/graph"
 KERNEL_OF_STAGE = {"init": "k_init", "populate1": "k_populate<1>", "rounds1": "k_rounds<1>",
@@ -455,7 +457,8 @@ def main():
                          "between steps"},
         "ms_per_graph": ms_max, "ms_per_step_all": per_step, "wall_s": wall,
         "edges_per_s_undirected": st["canonical_edges"] / (ms_max / 1e3),
-        "gpu_launches": args.steps * (LAUNCHES_PER_STEP if not use_dist else 4 + 4 * st["rounds"]),
+        "gpu_launches": args.steps * ((LAUNCHES_FILTERED if M >= 4 * n else LAUNCHES_UNFILTERED)
+                                      if not use_dist else 4 + 4 * st["rounds"]),
         "clocks": clocks,
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                      "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,

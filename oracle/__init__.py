@@ -45,6 +45,11 @@ def _load():
                                            ctypes.c_void_p, ctypes.c_void_p,
                                            ctypes.POINTER(ctypes.c_int64),
                                            ctypes.POINTER(ctypes.c_int64)]
+            lib.oracle_components.restype = ctypes.c_int64
+            lib.oracle_components.argtypes = [ctypes.c_int32, ctypes.c_void_p, ctypes.c_void_p]
+            lib.oracle_edge_in_msf.restype = ctypes.c_int
+            lib.oracle_edge_in_msf.argtypes = [ctypes.c_int32, ctypes.c_void_p, ctypes.c_void_p,
+                                               ctypes.c_void_p, ctypes.c_int64]
             _lib = lib
     return _lib
 
@@ -67,6 +72,28 @@ def kruskal(n, nindex, nlist, eweight):
     if rc != 0:
         raise ValueError(f"oracle_kruskal rejected the input (rc={rc})")
     return mask, int(total.value), int(count.value)
+
+
+def components(n, nindex, nlist):
+    """Number of connected components (one union-find scan of the CSR)."""
+    nindex = np.ascontiguousarray(nindex, dtype=np.int64)
+    nlist = np.ascontiguousarray(nlist, dtype=np.int32)
+    c = _load().oracle_components(int(n), nindex.ctypes.data, nlist.ctypes.data)
+    if c < 0:
+        raise ValueError("oracle_components rejected the input")
+    return int(c)
+
+
+def edge_in_msf(n, nindex, nlist, eweight, edge_id):
+    """Is canonical CSR entry edge_id in the MSF? (cycle-property definition)."""
+    nindex = np.ascontiguousarray(nindex, dtype=np.int64)
+    nlist = np.ascontiguousarray(nlist, dtype=np.int32)
+    eweight = np.ascontiguousarray(eweight, dtype=np.int32)
+    r = _load().oracle_edge_in_msf(int(n), nindex.ctypes.data, nlist.ctypes.data, eweight.ctypes.data,
+                                   int(edge_id))
+    if r < 0:
+        raise ValueError(f"entry {edge_id} is not a canonical edge")
+    return bool(r)
 
 
 def kruskal_graph(g):

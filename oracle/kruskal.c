@@ -117,3 +117,65 @@ int oracle_kruskal(int32_t n, const int64_t *nindex, const int32_t *nlist,
     if (count_out) *count_out = count;
     return 0;
 }
+
+/*
+ * Connected components of the graph (all canonical edges), by one scan of the
+ * CSR with the same disjoint-set forest.  Returns the number of components
+ * (>= 0) or -1 on invalid input.  An MSF has exactly n - #CC edges (P:63 fn 1).
+ */
+int64_t oracle_components(int32_t n, const int64_t *nindex, const int32_t *nlist)
+{
+    if (n < 0 || (n > 0 && !nindex)) return -1;
+    int32_t *parent = (int32_t *)malloc((size_t)(n > 0 ? n : 1) * sizeof(int32_t));
+    if (!parent) return -1;
+    for (int32_t v = 0; v < n; ++v) parent[v] = v;
+    int64_t comps = n;
+    for (int32_t u = 0; u < n; ++u)
+        for (int64_t j = nindex[u]; j < nindex[u + 1]; ++j) {
+            const int32_t v = nlist[j];
+            if (v < 0 || v >= n) { free(parent); return -1; }
+            if (!(u < v)) continue;
+            int32_t a = ds_find(parent, u), b = ds_find(parent, v);
+            if (a == b) continue;
+            if (a < b) { int32_t t = a; a = b; b = t; }
+            parent[a] = b;
+            --comps;
+        }
+    free(parent);
+    return comps;
+}
+
+/*
+ * Is canonical edge `id` in the MSF?  The cycle-property characterisation
+ * written out: e = (u, v, w, id) is in the unique MSF under the (w, id) order
+ * iff u and v are NOT connected by canonical edges that precede e in that
+ * order.  One scan of the CSR unioning exactly those edges.  Returns 1, 0, or
+ * -1 if `id` is not a canonical entry / the input is invalid.
+ */
+int oracle_edge_in_msf(int32_t n, const int64_t *nindex, const int32_t *nlist,
+                       const int32_t *eweight, int64_t id)
+{
+    if (n <= 0 || !nindex || id < 0 || id >= nindex[n]) return -1;
+    int32_t eu = -1;
+    for (int32_t u = 0; u < n; ++u)               /* row of entry id (linear: plain) */
+        if (nindex[u] <= id && id < nindex[u + 1]) { eu = u; break; }
+    const int32_t ev = nlist[id];
+    if (eu < 0 || !(eu < ev)) return -1;
+    const int32_t ew = eweight[id];
+    int32_t *parent = (int32_t *)malloc((size_t)n * sizeof(int32_t));
+    if (!parent) return -1;
+    for (int32_t v = 0; v < n; ++v) parent[v] = v;
+    for (int32_t u = 0; u < n; ++u)
+        for (int64_t j = nindex[u]; j < nindex[u + 1]; ++j) {
+            const int32_t v = nlist[j];
+            if (!(u < v)) continue;
+            const int32_t w = eweight[j];
+            const int lighter = (w < ew) || (w == ew && (uint64_t)j < (uint64_t)id);
+            if (!lighter) continue;
+            int32_t a = ds_find(parent, u), b = ds_find(parent, v);
+            if (a != b) parent[a] = b;
+        }
+    const int in = ds_find(parent, eu) != ds_find(parent, ev);
+    free(parent);
+    return in;
+}

@@ -13,7 +13,13 @@
 
 namespace eclmst {
 
-constexpr int kBlock = 512;                  // threads per CTA
+#ifndef ECL_R_BLOCK
+#define ECL_R_BLOCK 512
+#endif
+#ifndef ECL_R_MINB
+#define ECL_R_MINB 2
+#endif
+constexpr int kBlock = ECL_R_BLOCK;          // threads per k_rounds CTA
 constexpr int kWarps = kBlock / 32;
 constexpr int kItems = 4;                    // tuples / CSR entries per lane per warp chunk
 constexpr int kChunk = 32 * kItems;          // 128 per warp chunk

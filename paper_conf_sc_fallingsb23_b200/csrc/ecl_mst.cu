@@ -489,23 +489,26 @@ __global__ void __launch_bounds__(256) k_flatten(Params P) {
 // A CTA's worklist as a sequence of 128-tuple chunks.  Right after populate
 // it is the CTA's share of the populate regions (regions b, b+G, ..., each a
 // dense run of region[w].x tuples; chunk j maps to a region by a binary
-// search over s_pre); after a pass A it is one compact run of cnt tuples.
-struct Src {
-    const int4* base;   // compact mode
+// search over the shared prefix s_pre) -- RegionSrc; after a pass A it is one
+// compact run of cnt tuples -- CompactSrc.  Two types, so each pass is
+// compiled once per mode and carries only the registers that mode needs.
+struct CompactSrc {
+    const int4* base;
     int cnt;
-    int nloc;           // number of chunks
-    const int* s_pre;   // region mode (shared memory): chunk prefix per region, or null
-    const int* s_rcnt;  //   tuples per region
+    int nloc;
+    __device__ __forceinline__ const int4* get(const Params&, int j, int& count) const {
+        count = min(kChunk, cnt - j * kChunk);
+        return base + (long long)j * kChunk;
+    }
+};
+
+struct RegionSrc {
+    const int* s_pre;   // shared memory: chunk prefix per region (nreg + 1)
+    const int* s_rcnt;  // shared memory: tuples per region
     int nreg;
-    const int4* wl0;
-    long long rcap;
+    int nloc;
     int first_w;
-    int G;
-    __device__ __forceinline__ const int4* get(int j, int& count) const {
-        if (!s_pre) {
-            count = min(kChunk, cnt - j * kChunk);
-            return base + (long long)j * kChunk;
-        }
+    __device__ __forceinline__ const int4* get(const Params& P, int j, int& count) const {
         int lo = 0, hi = nreg;
         while (hi - lo > 1) {
             const int mid = (lo + hi) >> 1;
@@ -514,27 +517,73 @@ struct Src {
         }
         const int off = j - s_pre[lo];
         count = min(kChunk, s_rcnt[lo] - off * kChunk);
-        return wl0 + (long long)(first_w + lo * G) * rcap + (long long)off * kChunk;
+        return P.wl0 + (long long)(first_w + lo * P.G) * P.rcap + (long long)off * kChunk;
     }
 };
 
-__device__ __forceinline__ Src compact_src(const int4* base, int cnt) {
-    Src S;
+__device__ __forceinline__ CompactSrc compact_src(const int4* base, int cnt) {
+    CompactSrc S;
     S.base = base;
     S.cnt = cnt;
     S.nloc = (cnt + kChunk - 1) / kChunk;
-    S.s_pre = nullptr;
-    S.s_rcnt = nullptr;
-    S.nreg = 0;
-    S.wl0 = nullptr;
-    S.rcap = 0;
-    S.first_w = 0;
-    S.G = 0;
     return S;
 }
 
+// the populate output of CTA b: regions w = b, b + G, ...  Loads the region
+// counts into shared memory, builds the chunk prefix, and adds the kept,
+// canonical and deferred counts to the stats (phase 1 counters only if
+// count_phase1).  Every thread of the CTA must call it.
+__device__ __forceinline__ RegionSrc region_src(const Params& P, int b, int* s_pre, int* s_rcnt,
+                                                long long (*s_red)[kWarps], int64_t* live_slot,
+                                                bool count_phase1) {
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    RegionSrc R;
+    R.s_pre = s_pre;
+    R.s_rcnt = s_rcnt;
+    R.nreg = b < P.W ? (P.W - b + P.G - 1) / P.G : 0;
+    R.first_w = b;
+    long long canon = 0, heavy = 0;
+    for (int k = tid; k < R.nreg; k += kBlock) {
+        const int4 r = P.region[b + k * P.G];
+        s_rcnt[k] = r.x;
+        canon += r.y;
+        heavy += r.z;
+    }
+    canon = warp_sum(canon);
+    heavy = warp_sum(heavy);
+    if (lane == 0) {
+        s_red[1][warp] = canon;
+        s_red[2][warp] = heavy;
+    }
+    __syncthreads();
+    if (tid == 0) {
+        long long kept = 0;
+        int pre = 0;
+        for (int k = 0; k < R.nreg; ++k) {
+            s_pre[k] = pre;
+            pre += (s_rcnt[k] + kChunk - 1) / kChunk;
+            kept += s_rcnt[k];
+        }
+        s_pre[R.nreg] = pre;
+        canon = heavy = 0;
+        for (int w2 = 0; w2 < kWarps; ++w2) {
+            canon += s_red[1][w2];
+            heavy += s_red[2][w2];
+        }
+        if (kept) atomicAdd(reinterpret_cast<unsigned long long*>(live_slot), (unsigned long long)kept);
+        if (count_phase1) {
+            if (canon) atomicAdd(reinterpret_cast<unsigned long long*>(&P.st->canonical_edges), (unsigned long long)canon);
+            if (heavy) atomicAdd(reinterpret_cast<unsigned long long*>(&P.st->heavy_edges), (unsigned long long)heavy);
+        }
+    }
+    __syncthreads();
+    R.nloc = s_pre[R.nreg];
+    return R;
+}
+
 // L14-23 of one round over the CTA's worklist: S -> out (compact).
-__device__ __forceinline__ void passA(const Params& P, const Src& S, int4* __restrict__ out, int* s_out,
+template <class SRC>
+__device__ __forceinline__ void passA(const Params& P, const SRC& S, int4* __restrict__ out, int* s_out,
                                       bool guard) {
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const bool halving = P.halving != 0;
@@ -542,7 +591,7 @@ __device__ __forceinline__ void passA(const Params& P, const Src& S, int4* __res
     long long* __restrict__ K = P.key;
     for (int k = warp; k < S.nloc; k += kWarps) {
         int count;
-        const int4* __restrict__ in = S.get(k, count);
+        const int4* __restrict__ in = S.get(P, k, count);
         int4 t[kItems];
         bool keep[kItems];
 #pragma unroll
@@ -582,13 +631,14 @@ __device__ __forceinline__ void passA(const Params& P, const Src& S, int4* __res
 }
 
 // L27-31 (+ L34-37): check, join, mark over the CTA's worklist.
-__device__ __forceinline__ void passB(const Params& P, const Src& S, long long& wsum, long long& wcnt) {
+template <class SRC>
+__device__ __forceinline__ void passB(const Params& P, const SRC& S, long long& wsum, long long& wcnt) {
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     int* __restrict__ parent = P.parent;
     long long* __restrict__ K = P.key;
     for (int k = warp; k < S.nloc; k += kWarps) {
         int count;
-        const int4* __restrict__ in = S.get(k, count);
+        const int4* __restrict__ in = S.get(P, k, count);
         int4 t[kItems];
         bool ok[kItems];
 #pragma unroll
@@ -640,7 +690,7 @@ __device__ __forceinline__ bool use_guard(const Params& P, long long live, long 
 }
 
 template <int PH>
-__global__ void __launch_bounds__(kBlock, 2) k_rounds(Params P) {
+__global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
     cg::grid_group grid = cg::this_grid();
     __shared__ int s_out;
     __shared__ long long s_red[3][kWarps];
@@ -659,62 +709,17 @@ __global__ void __launch_bounds__(kBlock, 2) k_rounds(Params P) {
     const int b = blockIdx.x;
     int4* wl[2] = {P.wl0 + (long long)b * P.cap, P.wl1 + (long long)b * P.cap};
     // the populate output of this CTA: regions w = b, b + G, ... (region mode)
-    Src S;
-    S.base = nullptr;
-    S.cnt = 0;
-    S.s_pre = s_pre;
-    S.s_rcnt = s_rcnt;
-    S.nreg = b < P.W ? (P.W - b + P.G - 1) / P.G : 0;
-    S.wl0 = P.wl0;
-    S.rcap = P.rcap;
-    S.first_w = b;
-    S.G = P.G;
-    {
-        long long canon = 0, heavy = 0;
-        for (int k = tid; k < S.nreg; k += kBlock) {
-            const int4 r = P.region[b + k * P.G];
-            s_rcnt[k] = r.x;
-            canon += r.y;
-            heavy += r.z;
-        }
-        canon = warp_sum(canon);
-        heavy = warp_sum(heavy);
-        if (lane == 0) {
-            s_red[1][warp] = canon;
-            s_red[2][warp] = heavy;
-        }
-        __syncthreads();
-        if (tid == 0) {
-            long long kept = 0;
-            int pre = 0;
-            for (int k = 0; k < S.nreg; ++k) {
-                s_pre[k] = pre;
-                pre += (s_rcnt[k] + kChunk - 1) / kChunk;
-                kept += s_rcnt[k];
-            }
-            s_pre[S.nreg] = pre;
-            canon = heavy = 0;
-            for (int w2 = 0; w2 < kWarps; ++w2) {
-                canon += s_red[1][w2];
-                heavy += s_red[2][w2];
-            }
-            if (kept) atomicAdd(reinterpret_cast<unsigned long long*>(&st->live[g]), (unsigned long long)kept);
-            if (PH == 1) {
-                if (canon) atomicAdd(reinterpret_cast<unsigned long long*>(&st->canonical_edges), (unsigned long long)canon);
-                if (heavy) atomicAdd(reinterpret_cast<unsigned long long*>(&st->heavy_edges), (unsigned long long)heavy);
-            }
-            if (b0 && PH == 2) st->phase2_round = g;
-        }
-        __syncthreads();
-        S.nloc = s_pre[S.nreg];
-    }
+    const RegionSrc R = region_src(P, b, s_pre, s_rcnt, s_red, &st->live[g], PH == 1);
+    if (b0 && tid == 0 && PH == 2) st->phase2_round = g;
     trace_cta(P, 4 + 2 * g);
     grid.sync();
     long long wsum = 0, wcnt = 0;
     int cur = 0;
     bool overflow = false;
     long long L = __ldcg(&st->live[g]);
-    while (L > 0) {
+    CompactSrc C = compact_src(wl[0], 0);
+    // one round: pass B over S, then pass A from S into the other worklist
+    auto round = [&](const auto& S) {
         const long long w0 = wcnt;
         passB(P, S, wsum, wcnt);
         const long long d = warp_sum(wcnt - w0);
@@ -723,19 +728,26 @@ __global__ void __launch_bounds__(kBlock, 2) k_rounds(Params P) {
         trace_cta(P, 5 + 2 * g);
         grid.sync();
         stamp(P, 5 + 2 * g);
-        if (g + 1 >= ECL_MST_MAX_ROUNDS) { overflow = true; break; }
+        if (g + 1 >= ECL_MST_MAX_ROUNDS) {
+            overflow = true;
+            return false;
+        }
         const bool guard = use_guard(P, L, __ldcg(&st->winners[g]));
         ++g;
         passA(P, S, wl[cur ^ 1], &s_out, guard);
         cur ^= 1;
         __syncthreads();
-        S = compact_src(wl[cur], s_out);
-        if (tid == 0 && S.cnt) atomicAdd(reinterpret_cast<unsigned long long*>(&st->live[g]), (unsigned long long)S.cnt);
+        C = compact_src(wl[cur], s_out);
+        if (tid == 0 && C.cnt) atomicAdd(reinterpret_cast<unsigned long long*>(&st->live[g]), (unsigned long long)C.cnt);
         trace_cta(P, 4 + 2 * g);
         grid.sync();
         stamp(P, 4 + 2 * g);
         L = __ldcg(&st->live[g]);
-    }
+        return true;
+    };
+    if (L > 0 && round(R))
+        while (L > 0 && round(C)) {
+        }
     const long long s = warp_sum(wsum), c = warp_sum(wcnt);
     if (lane == 0) {
         if (s) atomicAdd(reinterpret_cast<unsigned long long*>(&st->total_weight), (unsigned long long)s);
@@ -852,59 +864,14 @@ __global__ void __launch_bounds__(kBlock, 2) k_dist_passA(Params P, int g, int c
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int b = blockIdx.x;
     int4* wl[2] = {P.wl0 + (long long)b * P.cap, P.wl1 + (long long)b * P.cap};
-    Src S;
-    if (FIRST) {
-        S.base = nullptr;
-        S.cnt = 0;
-        S.s_pre = s_pre;
-        S.s_rcnt = s_rcnt;
-        S.nreg = b < P.W ? (P.W - b + P.G - 1) / P.G : 0;
-        S.wl0 = P.wl0;
-        S.rcap = P.rcap;
-        S.first_w = b;
-        S.G = P.G;
-        long long canon = 0, heavy = 0;
-        for (int k = tid; k < S.nreg; k += kBlock) {
-            const int4 r = P.region[b + k * P.G];
-            s_rcnt[k] = r.x;
-            canon += r.y;
-            heavy += r.z;
-        }
-        canon = warp_sum(canon);
-        heavy = warp_sum(heavy);
-        if (lane == 0) {
-            s_red[1][warp] = canon;
-            s_red[2][warp] = heavy;
-        }
-        __syncthreads();
-        if (tid == 0) {
-            long long kept = 0;
-            int pre = 0;
-            for (int k = 0; k < S.nreg; ++k) {
-                s_pre[k] = pre;
-                pre += (s_rcnt[k] + kChunk - 1) / kChunk;
-                kept += s_rcnt[k];
-            }
-            s_pre[S.nreg] = pre;
-            canon = heavy = 0;
-            for (int w2 = 0; w2 < kWarps; ++w2) {
-                canon += s_red[1][w2];
-                heavy += s_red[2][w2];
-            }
-            if (kept) atomicAdd(reinterpret_cast<unsigned long long*>(&P.st->live[g - 1]), (unsigned long long)kept);
-            if (g - 1 == 0) {   // phase 1: |E| and the deferred count
-                if (canon) atomicAdd(reinterpret_cast<unsigned long long*>(&P.st->canonical_edges), (unsigned long long)canon);
-                if (heavy) atomicAdd(reinterpret_cast<unsigned long long*>(&P.st->heavy_edges), (unsigned long long)heavy);
-            }
-        }
-        __syncthreads();
-        S.nloc = s_pre[S.nreg];
-    } else {
-        S = compact_src(wl[cur], P.acnt[b]);
-    }
     if (tid == 0) s_out = 0;
-    __syncthreads();
-    passA(P, S, wl[cur ^ 1], &s_out, P.guards != 0);
+    if (FIRST) {
+        const RegionSrc R = region_src(P, b, s_pre, s_rcnt, s_red, &P.st->live[g - 1], g - 1 == 0);
+        passA(P, R, wl[cur ^ 1], &s_out, P.guards != 0);
+    } else {
+        __syncthreads();
+        passA(P, compact_src(wl[cur], P.acnt[b]), wl[cur ^ 1], &s_out, P.guards != 0);
+    }
     __syncthreads();
     if (tid == 0) {
         P.acnt[b] = s_out;
@@ -1125,18 +1092,21 @@ int ecl_mst_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t* n
     if (e == cudaSuccess)
         e = cudaLaunchCooperativeKernel(reinterpret_cast<const void*>(k_rounds<1>), dim3((unsigned)G), dim3(kBlock), args, 0, s);
     if (e == cudaSuccess) e = mark();
-    if (e == cudaSuccess) {
+    // phase 2 can only happen when filtering is on; with the automatic rule
+    // (M >= 4n) the host knows that already and skips the three launches
+    const bool maybe_phase2 = P.filter_mode > 0 || (P.filter_mode < 0 && M >= 4LL * n);
+    if (e == cudaSuccess && maybe_phase2) {
         k_flatten<1><<<flat_blocks, 256, 0, s>>>(P);
         k_flatten<2><<<flat_blocks, 256, 0, s>>>(P);
         e = cudaGetLastError();
     }
     if (e == cudaSuccess) e = mark();
-    if (e == cudaSuccess) {
+    if (e == cudaSuccess && maybe_phase2) {
         k_populate<2><<<(unsigned)pop_blocks, kPopBlock, 0, s>>>(P);
         e = cudaGetLastError();
     }
     if (e == cudaSuccess) e = mark();
-    if (e == cudaSuccess)
+    if (e == cudaSuccess && maybe_phase2)
         e = cudaLaunchCooperativeKernel(reinterpret_cast<const void*>(k_rounds<2>), dim3((unsigned)G), dim3(kBlock), args, 0, s);
     if (e == cudaSuccess) e = mark();
     if (e == cudaSuccess) {

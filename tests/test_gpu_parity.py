@@ -185,3 +185,51 @@ def test_full_size_exact(eclmst, name):
     g = synth.make_config(name, "full", device="cuda:0").to("cpu")
     stats = assert_parity(eclmst, g)
     check_round_bound(g, stats)
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("name", ["rgg", "rmat"])
+def test_full_size_exact_large(eclmst, name):
+    """BASELINE configs C3/C4 at full size (100M / 521M CSR entries), whole
+    mask vs the oracle (the C4 oracle run takes about a minute)."""
+    g = synth.make_config(name, "full", device="cuda:0").to("cpu")
+    stats = assert_parity(eclmst, g)
+    check_round_bound(g, stats)
+
+
+@pytest.mark.slow
+def test_full_size_c5_sampled(eclmst):
+    """C5 at full size (n = 2^26, M = 2.0e9): a whole serial Kruskal would need
+    minutes and 40 GB, so check what holds at any size -- the forest has
+    n - #CC edges (#CC by the oracle's union-find scan), only canonical slots
+    are marked, the total is the sum of the marked weights -- and decide
+    sampled edges one by one with the oracle's cycle-property definition."""
+    gd = synth.make_config("uniform", "full", device="cuda:0")
+    mask_d, total_d, ws = eclmst.ecl_mst_device(gd.n, gd.nindex, gd.nlist, gd.eweight)
+    st = eclmst.ecl_mst_read_stats(ws)
+    assert st["status"] == 0
+    n = gd.n
+    nindex = gd.nindex.cpu().numpy()
+    nlist = gd.nlist.cpu().numpy()
+    eweight = gd.eweight.cpu().numpy()
+    mask = mask_d.cpu().numpy()
+    del gd
+    total = int(total_d.item())
+    ncc = oracle.components(n, nindex, nlist)
+    marked = np.flatnonzero(mask)
+    assert len(marked) == n - ncc == st["msf_edges"]
+    rows = np.searchsorted(nindex, marked, side="right") - 1
+    assert np.all(rows < nlist[marked])                      # canonical slots only
+    assert int(eweight[marked].astype(np.int64).sum()) == total
+    # sample among the lighter edges: each one-by-one decision scans only the
+    # edges that precede it, so light samples keep the check to seconds
+    rng = np.random.default_rng(11)
+    light = np.int32(1 << 27)                                  # weights are uniform in [0, 2^31)
+    lm = marked[eweight[marked] < light]
+    picks = [int(j) for j in rng.choice(lm, 3, replace=False)]
+    tries = rng.integers(0, len(nlist), 4096)
+    trows = np.searchsorted(nindex, tries, side="right") - 1
+    unmarked = [int(j) for j, r in zip(tries, trows) if r < nlist[j] and not mask[j] and eweight[j] < light][:3]
+    assert len(unmarked) == 3
+    for j in picks + unmarked:
+        assert oracle.edge_in_msf(n, nindex, nlist, eweight, int(j)) == bool(mask[j]), j

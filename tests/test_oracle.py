@@ -194,3 +194,23 @@ def test_rng_matches_scalar_splitmix():
     for i, x in zip(idx.tolist(), h.tolist()):
         assert (x & ((1 << 64) - 1)) == synth.rng.hash_u64_py(12, 5, i)
     assert synth.splitmix64_py(0) == 0xE220A8397B1DCDAF   # published splitmix64 first output
+
+
+# --- the per-edge and component helpers used for full-size (sampled) checks ---
+
+@pytest.mark.parametrize("seed", range(6))
+def test_edge_in_msf_and_components_agree_with_pins(seed):
+    kinds = ["ties", "two", "full", "uniform", "equal", "ties"]
+    g = G.random_small(60 + seed, 150, seed=300 + seed, weights=kinds[seed], multi=seed % 2 == 0,
+                       self_loops=seed % 3 == 0)
+    n, nindex, nlist, eweight = g.numpy()
+    u, v, w, ids = refs.canonical_edges(n, nindex, nlist, eweight)
+    cmask = refs.lighter_path_msf(n, nindex, nlist, eweight)     # independent BFS characterisation
+    for j in ids.tolist():
+        assert oracle.edge_in_msf(n, nindex, nlist, eweight, j) == bool(cmask[j])
+    ncc, _ = refs.components(n, u, v)
+    assert oracle.components(n, nindex, nlist) == ncc
+    with pytest.raises(ValueError):
+        rows = np.repeat(np.arange(n), np.diff(nindex))
+        mirror = int(np.nonzero(rows > nlist)[0][0])
+        oracle.edge_in_msf(n, nindex, nlist, eweight, mirror)
