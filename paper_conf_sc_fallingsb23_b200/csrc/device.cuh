@@ -26,6 +26,16 @@ constexpr int kChunk = 32 * kItems;          // 128 per warp chunk
 constexpr long long kInf = LLONG_MAX;        // "no edge recorded" (reading Q4)
 constexpr unsigned kFull = 0xffffffffu;
 
+// View of the per-vertex state: disjoint-set parent and best-edge key
+// (minEdge), two arrays.  (Interleaving them into 16-byte records was
+// measured slower on every config: C5 86.9 vs 73.9 ms, road 2.92 vs 2.38 ms.)
+struct DS {
+    int* parent;
+    long long* key;
+    __device__ __forceinline__ int* par(long long v) const { return parent + v; }
+    __device__ __forceinline__ long long* k(long long v) const { return key + v; }
+};
+
 // (weight:id) key, weight in the most significant bits: signed order
 // of the key == lexicographic order of (weight as int32, id as uint32).
 __device__ __forceinline__ long long make_key(int w, unsigned id) {
@@ -52,19 +62,19 @@ __device__ __forceinline__ unsigned long long globaltimer_ns() {
 // Continue a find() from x whose parent px is already loaded.  With halving
 // on, every visited non-root is re-pointed to its grandparent (path halving;
 // a benign race: the stored value is always an ancestor).
-__device__ __forceinline__ int find_from(int* __restrict__ parent, int x, int px, bool halving) {
+__device__ __forceinline__ int find_from(const DS& D, int x, int px, bool halving) {
     while (px != x) {
-        const int ppx = __ldca(parent + px);
+        const int ppx = __ldca(D.par(px));
         if (ppx == px) return px;
-        if (halving) parent[x] = ppx;
+        if (halving) *D.par(x) = ppx;
         x = ppx;
-        px = __ldca(parent + x);
+        px = __ldca(D.par(x));
     }
     return x;
 }
 
-__device__ __forceinline__ int find_root(int* __restrict__ parent, int x, bool halving) {
-    return find_from(parent, x, __ldca(parent + x), halving);
+__device__ __forceinline__ int find_root(const DS& D, int x, bool halving) {
+    return find_from(D, x, __ldca(D.par(x)), halving);
 }
 
 // 64-bit atomicMin (L20-21) with the paper's optional guard: a plain

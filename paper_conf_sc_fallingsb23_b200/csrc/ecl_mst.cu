@@ -66,11 +66,12 @@ struct Internal {
     unsigned int done;                 // unused ticket
     int g_cur;                         // first global round of the running phase
     int g_end;                         // last global round of the finished phase
+    int giant;                         // root of the largest set after phase 1 (-1: none)
     int pad0;
 };
 
 struct Layout {
-    size_t stats, internal, trace, rowstart, region, key, parent, wl0, wl1, total;
+    size_t stats, internal, trace, rowstart, region, giant, key, parent, wl0, wl1, total;
     long long wl_cap;                  // tuples per worklist buffer
 };
 
@@ -96,6 +97,7 @@ static inline Layout layout_for(int64_t n, int64_t M) {
     L.trace = off;    off = align_up(off + sizeof(long long) * kTraceSlots * kMaxGrid, 256);
     L.rowstart = off; off = align_up(off + sizeof(int) * (size_t)(nchunks + 1), 256);
     L.region = off;   off = align_up(off + sizeof(int4) * (size_t)kMaxPopWarps, 256);
+    L.giant = off;    off = align_up(off + sizeof(unsigned) * (size_t)((n + 31) / 32 + 1), 256);
     L.key = off;      off = align_up(off + sizeof(long long) * (size_t)n, 256);
     L.parent = off;   off = align_up(off + sizeof(int) * (size_t)n, 256);
     L.wl0 = off;      off = align_up(off + sizeof(int4) * (size_t)L.wl_cap, 256);
@@ -122,6 +124,7 @@ struct Params {
     long long* trace;                 // [kTraceSlots][kMaxGrid] or null
     int* rowstart;                    // row of CSR entry c*kChunk, per chunk
     int4* region;                     // per populate warp: {tuples, canonical, heavy, 0}
+    unsigned* giant_bits;             // bit v: v is in the largest set after phase 1 (or null)
     long long* key;
     int* parent;
     int4* wl0;
@@ -144,6 +147,13 @@ struct Params {
     long long* const* keys_all;       // virtual shards: every shard's key array
     int nkeys;
 };
+
+__device__ __forceinline__ DS ds_of(const Params& P) {
+    DS D;
+    D.parent = P.parent;
+    D.key = P.key;
+    return D;
+}
 
 __device__ __forceinline__ void stamp(const Params& P, int slot) {
     if (blockIdx.x == 0 && threadIdx.x == 0 && slot < kTraceSlots)
@@ -225,6 +235,7 @@ __global__ void __launch_bounds__(256) k_init(Params P) {
             P.in->g_cur = 0;
             P.in->g_end = 0;
             P.in->done = 0;
+            P.in->giant = -1;
         }
     }
     if (err) atomicExch(&P.st->status, ECL_MST_ERR_INPUT);
@@ -234,6 +245,15 @@ __global__ void __launch_bounds__(256) k_init(Params P) {
 // k_populate<PH>: one warp per 128-entry CSR chunk
 // ---------------------------------------------------------------------------
 template <int PH>
+#ifndef ECL_DEEP_PH1
+#define ECL_DEEP_PH1 0
+#endif
+#ifndef ECL_DEEP_PH2
+#define ECL_DEEP_PH2 1
+#endif
+#ifndef ECL_GIANT_MIN_N
+#define ECL_GIANT_MIN_N (32LL << 20)   // parent[] larger than ~half the L2
+#endif
 #ifndef ECL_POP_MINB
 #define ECL_POP_MINB 4
 #endif
@@ -248,8 +268,7 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
     const bool filtered = __ldg(&P.st->filtered) != 0;
     const int T = __ldg(&P.st->threshold);
     const bool guard = (P.guards > 0) || (P.guards < 0 && PH == 2);
-    long long* __restrict__ K = P.key;
-    int* __restrict__ parent = P.parent;
+    const DS D = ds_of(P);
     // warp w takes chunks w, w + W, ... (an even sample of the whole CSR, so
     // every region -- and every k_rounds CTA -- gets the same mix even where
     // the density of u < v entries drifts along the rows) and appends its
@@ -278,17 +297,47 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
             }
         }
     };
-    // software pipeline, one chunk ahead: the row bracket and the CSR entries
-    // of the next chunk are in flight while this one is processed (a deeper
-    // prefetch of the row starts measured no faster)
-    // (edge sharding: this shard owns chunks shard, shard + nshards, ...;
-    // lc indexes them, c is the global chunk)
-    int nr0 = 0, nrl = 0, nv[kItems], nw[kItems];
+    // software pipeline (edge sharding: this shard owns chunks shard,
+    // shard + nshards, ...; lc indexes them, c is the global chunk).  While
+    // chunk i is processed, chunk i+1's CSR entries and its first 64 row
+    // starts, and chunk i+2's row bracket, are in flight; at the end of
+    // chunk i the phase-2 membership bits of chunk i+1's far ends are
+    // requested (their entries have arrived by then).
+    const int giant = (PH == 2 && P.flatten && P.giant_bits) ? __ldg(&P.in->giant) : -1;
+    // deep: also prefetch the next chunk's row starts (phase 2, where the
+    // bitmap / parent loads already lengthen each chunk's chain)
+    constexpr bool deep = PH == 1 ? ECL_DEEP_PH1 : ECL_DEEP_PH2;
+    auto bracket = [&](long long lc, int& r0, int& rl) {
+        const long long c = P.shard + lc * P.nshards;
+        r0 = __ldg(P.rowstart + c);
+        rl = (c + 1 < P.nchunks) ? __ldg(P.rowstart + c + 1) : P.n - 1;
+    };
+    auto starts = [&](int r0, int rl, long long& sa, long long& sz) {
+        const int ra = r0 + 1 + lane, rz = r0 + 33 + lane;
+        sa = ra <= rl ? __ldg(P.nindex + ra) : LLONG_MAX;
+        sz = rz <= rl ? __ldg(P.nindex + rz) : LLONG_MAX;
+    };
+    auto vbits = [&](const int (&vv)[kItems]) {
+        unsigned b = 0;
+        if (PH == 2 && giant >= 0) {
+#pragma unroll
+            for (int k = 0; k < kItems; ++k)
+                if ((unsigned)vv[k] < (unsigned)P.n)
+                    b |= ((__ldg(P.giant_bits + (vv[k] >> 5)) >> (vv[k] & 31)) & 1u) << k;
+        }
+        return b;
+    };
+    int nr0 = 0, nrl = 0, n2r0 = 0, n2rl = 0, nv[kItems], nw[kItems];
+    long long nsa = LLONG_MAX, nsz = LLONG_MAX;
+    unsigned nvb = 0;
     if (w < P.nlocal) {
-        const long long c = P.shard + (long long)w * P.nshards;
-        nr0 = __ldg(P.rowstart + c);
-        nrl = (c + 1 < P.nchunks) ? __ldg(P.rowstart + c + 1) : P.n - 1;
-        load_entries(c, nv, nw);
+        bracket(w, nr0, nrl);
+        load_entries(P.shard + (long long)w * P.nshards, nv, nw);
+        if (deep) {
+            starts(nr0, nrl, nsa, nsz);
+            if (w + P.W < P.nlocal) bracket(w + P.W, n2r0, n2rl);
+        }
+        nvb = vbits(nv);
     }
     for (long long lc = w; lc < P.nlocal; lc += P.W) {
     const long long c = P.shard + lc * P.nshards;
@@ -302,6 +351,8 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
         const int len = (int)(c1 - c0);
         // rows of this chunk: r0 = row of entry c0; rows r0+1 .. r_last start inside
         const int r0 = nr0, r_last = nrl;
+        const long long sa = nsa, sz = nsz;
+        const unsigned vb = nvb;
         int vv[kItems], ww[kItems];
 #pragma unroll
         for (int k = 0; k < kItems; ++k) {
@@ -309,24 +360,36 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
             ww[k] = nw[k];
         }
         const long long lcn = lc + P.W;
-        const long long cn = P.shard + lcn * P.nshards;
         if (lcn < P.nlocal) {
-            nr0 = __ldg(P.rowstart + cn);
-            nrl = (cn + 1 < P.nchunks) ? __ldg(P.rowstart + cn + 1) : P.n - 1;
-            load_entries(cn, nv, nw);
+            load_entries(P.shard + lcn * P.nshards, nv, nw);
+            if (deep) {
+                nr0 = n2r0;
+                nrl = n2rl;
+                starts(nr0, nrl, nsa, nsz);
+                if (lcn + P.W < P.nlocal) bracket(lcn + P.W, n2r0, n2rl);
+            } else {
+                bracket(lcn, nr0, nrl);
+            }
         }
         int* mark = s_mark[warp];
 #pragma unroll
         for (int i = lane; i < kChunk; i += 32) mark[i] = -1;
         __syncwarp();
-        for (int rb = r0 + 1; rb <= r_last; rb += 64) {   // two independent batches of row starts
-            const int ra = rb + lane, rz = rb + 32 + lane;
-            const long long sa = ra <= r_last ? __ldg(P.nindex + ra) : LLONG_MAX;
-            const long long sz = rz <= r_last ? __ldg(P.nindex + rz) : LLONG_MAX;
+        if (deep) {   // the first 64 row starts arrived with the prefetch
+            const int ra = r0 + 1 + lane, rz = r0 + 33 + lane;
             if (sa >= c0 && sa < c1) atomicMax(&mark[sa - c0], ra);
             else if (sa < c0) err = true;
             if (sz >= c0 && sz < c1) atomicMax(&mark[sz - c0], rz);
             else if (sz < c0) err = true;
+        }
+        for (int rb = r0 + (deep ? 65 : 1); rb <= r_last; rb += 64) {   // (further) row starts
+            const int ra = rb + lane, rz = rb + 32 + lane;
+            const long long ta = ra <= r_last ? __ldg(P.nindex + ra) : LLONG_MAX;
+            const long long tz = rz <= r_last ? __ldg(P.nindex + rz) : LLONG_MAX;
+            if (ta >= c0 && ta < c1) atomicMax(&mark[ta - c0], ra);
+            else if (ta < c0) err = true;
+            if (tz >= c0 && tz < c1) atomicMax(&mark[tz - c0], rz);
+            else if (tz < c0) err = true;
         }
         __syncwarp();
         int row[kItems];
@@ -380,9 +443,12 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
         if (PH == 2) {   // set(v), set(n): one load each after k_flatten
 #pragma unroll
             for (int k = 0; k < kItems; ++k) {
-                if (cand[k]) {
-                    pk[k] = (k > 0 && cand[k - 1] && row[k] == row[k - 1]) ? -1 : __ldca(parent + row[k]);
-                    qk[k] = __ldca(parent + vv[k]);
+                if (cand[k] && giant >= 0 && ((vb >> k) & 1u) &&
+                    ((__ldg(P.giant_bits + (row[k] >> 5)) >> (row[k] & 31)) & 1)) {
+                    pk[k] = qk[k] = giant;                    // both ends in the largest set: filtered
+                } else if (cand[k]) {
+                    pk[k] = (k > 0 && cand[k - 1] && row[k] == row[k - 1]) ? -1 : __ldca(D.par(row[k]));
+                    qk[k] = __ldca(D.par(vv[k]));
                 }
             }
 #pragma unroll
@@ -392,8 +458,8 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
 #pragma unroll
                 for (int k = 0; k < kItems; ++k) {
                     if (cand[k]) {
-                        pk[k] = find_root(parent, pk[k], P.halving != 0);
-                        qk[k] = find_root(parent, qk[k], P.halving != 0);
+                        pk[k] = find_root(D, pk[k], P.halving != 0);
+                        qk[k] = find_root(D, qk[k], P.halving != 0);
                     }
                 }
             }
@@ -412,18 +478,19 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
             if (!keep[k]) continue;
             const long long key = make_key(t[k].z, (unsigned)t[k].w);   // L19 val <- e_w : e_id
             if (t[k].x != bp) {
-                if (bp >= 0) record_min(K + bp, best, guard);
+                if (bp >= 0) record_min(D.k(bp), best, guard);
                 bp = t[k].x;
                 best = key;
             } else {
                 best = min(best, key);
             }
         }
-        if (bp >= 0) record_min(K + bp, best, guard);
+        if (bp >= 0) record_min(D.k(bp), best, guard);
 #pragma unroll
         for (int k = 0; k < kItems; ++k)
-            if (keep[k]) record_min(K + t[k].y, make_key(t[k].z, (unsigned)t[k].w), guard);
+            if (keep[k]) record_min(D.k(t[k].y), make_key(t[k].z, (unsigned)t[k].w), guard);
     }
+    if (PH == 2 && lc + P.W < P.nlocal) nvb = vbits(nv);   // next chunk's far-end bits
     // L7: append the chunk's tuples to the warp's region
     unsigned m[kItems];
     int off[kItems];
@@ -462,23 +529,60 @@ template <int STAGE>
 __global__ void __launch_bounds__(256) k_flatten(Params P) {
     if (!phase2_needed(P) || !P.flatten) return;
     const long long stride = (long long)gridDim.x * blockDim.x;
-    int* __restrict__ parent = P.parent;
-    for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < P.n; v += stride) {
+    const DS D = ds_of(P);
+    const int lane = threadIdx.x & 31;
+    const int giant = (STAGE == 2 && P.giant_bits) ? __ldcg(&P.in->giant) : -1;
+    // warps walk 32 consecutive vertices together (stage 2 ballots the bitmap)
+    for (long long base = (long long)blockIdx.x * blockDim.x + threadIdx.x - lane; base < P.n; base += stride) {
+        const long long v = base + lane;
+        const bool valid = v < P.n;
         if (STAGE == 1) {
             // fast, racy compression: path halving by everybody (ends close
             // to, but not always exactly at, one hop)
-            const int r = find_root(parent, (int)v, true);
-            if (r != (int)v) parent[v] = r;
+            if (valid) {
+                const int r = find_root(D, (int)v, true);
+                if (r != (int)v) *D.par(v) = r;
+            }
         } else {
             // exact: owner-only pointer jumping over the now-short paths
-            int p = __ldcg(parent + v);
-            while (true) {
-                const int pp = __ldcg(parent + p);
+            int p = valid ? __ldcg(D.par(v)) : -1;
+            while (valid) {
+                const int pp = __ldcg(D.par(p));
                 if (pp == p) break;
-                __stcg(parent + v, pp);
+                __stcg(D.par(v), pp);
                 p = pp;
             }
+            if (P.giant_bits) {
+                const unsigned bits = __ballot_sync(kFull, valid && p == giant);
+                if (lane == 0) P.giant_bits[base >> 5] = bits;
+            }
         }
+    }
+}
+
+// After phase 1 most vertices of a graph whose light edges percolate (C3-C5)
+// sit in ONE set.  Find its root by a majority vote over sampled vertices;
+// k_flatten<2> then writes a bitmap of its members, and the phase-2 populate
+// filters an edge with both ends in it from the bitmap (n/8 bytes, L2
+// resident) instead of two random parent loads.
+__global__ void __launch_bounds__(256) k_giant(Params P) {
+    __shared__ int s_r[1024];
+    if (!phase2_needed(P) || !P.flatten || !P.giant_bits) return;
+    const DS D = ds_of(P);
+    for (int i = threadIdx.x; i < 1024; i += blockDim.x) {
+        const long long v = (long long)(splitmix64(0x6A09E667F3BCC909ull + (unsigned long long)i) % (unsigned long long)P.n);
+        s_r[i] = find_root(D, (int)v, false);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        int cand = -1, votes = 0;                 // Boyer-Moore majority vote
+        for (int i = 0; i < 1024; ++i) {
+            if (votes == 0) { cand = s_r[i]; votes = 1; }
+            else votes += (s_r[i] == cand) ? 1 : -1;
+        }
+        int cnt = 0;
+        for (int i = 0; i < 1024; ++i) cnt += s_r[i] == cand;
+        P.in->giant = cnt >= 256 ? cand : -1;     // worth a bitmap only if it holds >= 1/4
     }
 }
 
@@ -587,8 +691,7 @@ __device__ __forceinline__ void passA(const Params& P, const SRC& S, int4* __res
                                       bool guard) {
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const bool halving = P.halving != 0;
-    int* __restrict__ parent = P.parent;
-    long long* __restrict__ K = P.key;
+    const DS D = ds_of(P);
     for (int k = warp; k < S.nloc; k += kWarps) {
         int count;
         const int4* __restrict__ in = S.get(P, k, count);
@@ -604,15 +707,15 @@ __device__ __forceinline__ void passA(const Params& P, const SRC& S, int4* __res
 #pragma unroll
         for (int i = 0; i < kItems; ++i) {
             if (keep[i]) {
-                px[i] = __ldca(parent + t[i].x);
-                qx[i] = __ldca(parent + t[i].y);
+                px[i] = __ldca(D.par(t[i].x));
+                qx[i] = __ldca(D.par(t[i].y));
             }
         }
 #pragma unroll
         for (int i = 0; i < kItems; ++i) {
             if (keep[i]) {
-                const int p = find_from(parent, t[i].x, px[i], halving);   // L15
-                const int q = find_from(parent, t[i].y, qx[i], halving);   // L16
+                const int p = find_from(D, t[i].x, px[i], halving);        // L15
+                const int q = find_from(D, t[i].y, qx[i], halving);        // L16
                 keep[i] = p != q;                                          // L17
                 t[i].x = p;                                                // L18: implicit
                 t[i].y = q;                                                //      path compression
@@ -622,8 +725,8 @@ __device__ __forceinline__ void passA(const Params& P, const SRC& S, int4* __res
         for (int i = 0; i < kItems; ++i) {
             if (keep[i]) {
                 const long long key = make_key(t[i].z, (unsigned)t[i].w); // L19
-                record_min(K + t[i].x, key, guard);                       // L20
-                record_min(K + t[i].y, key, guard);                       // L21
+                record_min(D.k(t[i].x), key, guard);                      // L20
+                record_min(D.k(t[i].y), key, guard);                      // L21
             }
         }
         warp_emit(t, keep, out, s_out);                                   // L18
@@ -634,8 +737,7 @@ __device__ __forceinline__ void passA(const Params& P, const SRC& S, int4* __res
 template <class SRC>
 __device__ __forceinline__ void passB(const Params& P, const SRC& S, long long& wsum, long long& wcnt) {
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    int* __restrict__ parent = P.parent;
-    long long* __restrict__ K = P.key;
+    const DS D = ds_of(P);
     for (int k = warp; k < S.nloc; k += kWarps) {
         int count;
         const int4* __restrict__ in = S.get(P, k, count);
@@ -651,13 +753,12 @@ __device__ __forceinline__ void passB(const Params& P, const SRC& S, long long& 
         // edge, so id equality is key equality (and inf's id half, 2^32-1,
         // is never a valid id).  L1 is fine: K[p] only changes when p's own
         // winner resets it.
-        const unsigned* __restrict__ Kid = reinterpret_cast<const unsigned*>(K);
         unsigned kp[kItems], kq[kItems];
 #pragma unroll
         for (int i = 0; i < kItems; ++i) {
             if (ok[i]) {
-                kp[i] = __ldca(Kid + 2 * (long long)t[i].x);
-                kq[i] = __ldca(Kid + 2 * (long long)t[i].y);
+                kp[i] = __ldca(reinterpret_cast<const unsigned*>(D.k(t[i].x)));
+                kq[i] = __ldca(reinterpret_cast<const unsigned*>(D.k(t[i].y)));
             }
         }
 #pragma unroll
@@ -668,10 +769,10 @@ __device__ __forceinline__ void passB(const Params& P, const SRC& S, long long& 
                 const int p = t[i].x, q = t[i].y;
                 // L30 join: each set hooks along its own lightest edge;
                 // a mutual pair keeps the smaller representative as root.
-                if (wp && !(wq && p < q)) __stcg(parent + p, q);
-                if (wq && !(wp && q < p)) __stcg(parent + q, p);
-                if (wp) __stcg(K + p, kInf);                           // L35
-                if (wq) __stcg(K + q, kInf);                           // L36
+                if (wp && !(wq && p < q)) __stcg(D.par(p), q);
+                if (wq && !(wp && q < p)) __stcg(D.par(q), p);
+                if (wp) __stcg(D.k(p), kInf);                          // L35
+                if (wq) __stcg(D.k(q), kInf);                          // L36
                 P.in_mst[(unsigned)t[i].w] = 1;                        // L31
                 wsum += t[i].z;
                 wcnt += 1;
@@ -810,13 +911,14 @@ __global__ void __launch_bounds__(256) k_dist_reps1(Params P) {
     const long long stride = (long long)gridDim.x * blockDim.x;
     unsigned long long found = 0;
     for (long long x = (long long)blockIdx.x * blockDim.x + threadIdx.x; x < P.n; x += stride) {
-        const long long kx = P.key[x];
+        const long long kx = P.key[x];   // distributed path: own arrays (stride 1)
         if (kx == kInf) continue;
         ++found;
         const unsigned j = (unsigned)(kx & 0xffffffffll);
         const int u = row_of_entry(P, (long long)j);
         const int v = __ldg(P.nlist + j);
-        const int pu = find_root(P.parent, u, false), pv = find_root(P.parent, v, false);
+        const DS D = ds_of(P);
+        const int pu = find_root(D, u, false), pv = find_root(D, v, false);
         const int q = (pu == (int)x) ? pv : pu;
         const bool mutual = P.key[q] == kx;
         P.tgt[x] = q | (mutual ? (int)0x80000000 : 0);
@@ -1034,6 +1136,8 @@ int ecl_mst_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t* n
     P.trace = o.trace ? reinterpret_cast<long long*>(ws + L.trace) : nullptr;
     P.rowstart = reinterpret_cast<int*>(ws + L.rowstart);
     P.region = reinterpret_cast<int4*>(ws + L.region);
+    // the largest-set bitmap only pays when parent[] does not fit the L2
+    P.giant_bits = (long long)n >= ECL_GIANT_MIN_N ? reinterpret_cast<unsigned*>(ws + L.giant) : nullptr;
     P.key = reinterpret_cast<long long*>(ws + L.key);
     P.parent = reinterpret_cast<int*>(ws + L.parent);
     P.wl0 = reinterpret_cast<int4*>(ws + L.wl0);
@@ -1097,6 +1201,7 @@ int ecl_mst_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t* n
     const bool maybe_phase2 = P.filter_mode > 0 || (P.filter_mode < 0 && M >= 4LL * n);
     if (e == cudaSuccess && maybe_phase2) {
         k_flatten<1><<<flat_blocks, 256, 0, s>>>(P);
+        k_giant<<<1, 256, 0, s>>>(P);
         k_flatten<2><<<flat_blocks, 256, 0, s>>>(P);
         e = cudaGetLastError();
     }
