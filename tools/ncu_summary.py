@@ -31,7 +31,7 @@ def stage_of(kernel_name):
                     ("k_populate<2>", "populate2"), ("k_populate<(int)2>", "populate2"),
                     ("k_rounds<1>", "rounds1"), ("k_rounds<(int)1>", "rounds1"),
                     ("k_rounds<2>", "rounds2"), ("k_rounds<(int)2>", "rounds2"),
-                    ("k_flatten", "flatten"), ("k_finalize", "finalize")):
+                    ("k_flatten", "flatten"), ("k_giant", "flatten"), ("k_finalize", "finalize")):
         if pat in k:
             return st
     return k
