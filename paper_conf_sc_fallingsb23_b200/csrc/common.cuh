@@ -1,0 +1,141 @@
+// common.cuh -- constants, workspace layout, kernel parameters and small
+// helpers shared by the kernels of the ECL-MST hot path (ecl_mst.cu).
+#pragma once
+
+#include <cooperative_groups.h>
+#include <cuda_runtime.h>
+
+#include <climits>
+#include <cstdint>
+
+#include "device.cuh"
+#include "ecl_mst.h"
+
+namespace cg = cooperative_groups;
+
+namespace eclmst {
+
+constexpr int kMaxGrid = 4096;                 // CTAs of k_rounds (= arenas), upper bound
+constexpr int kPopWarps = 8;                   // warps per k_populate CTA (one chunk each)
+constexpr int kPopBlock = 32 * kPopWarps;
+constexpr int kMaxPopWarps = 65536;            // populate warps (= worklist regions), upper bound
+constexpr int kMaxRegionsPerCta = 256;         // regions a k_rounds CTA starts from
+constexpr int kTraceSlots = 2 * ECL_MST_MAX_ROUNDS + 4;
+constexpr int kMaxSamples = 4096;              // threshold sample size cap
+static_assert(kMaxGrid == ECL_MST_TRACE_CTAS, "trace layout");
+
+struct Internal {
+    unsigned long long reps;           // distributed path: sets with a finite key this round
+    unsigned int done;                 // unused ticket
+    int g_cur;                         // first global round of the running phase
+    int g_end;                         // last global round of the finished phase
+    int giant;                         // root of the largest set after phase 1 (-1: none)
+    int pad0;
+};
+
+struct Layout {
+    size_t stats, internal, trace, rowstart, region, giant, key, parent, wl0, wl1, total;
+    long long wl_cap;                  // tuples per worklist buffer
+};
+
+static inline size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
+
+static inline long long ceil_div(long long a, long long b) { return (a + b - 1) / b; }
+
+// worklist tuples needed for W populate regions of ceil(nchunks/W)*kChunk
+// tuples, for any W <= min(kMaxPopWarps, nchunks)
+static inline long long wl_capacity(long long M) {
+    const long long nchunks = ceil_div(M, kChunk);
+    const long long wmax = nchunks < kMaxPopWarps ? nchunks : kMaxPopWarps;
+    return (nchunks + wmax) * (long long)kChunk;
+}
+
+static inline Layout layout_for(int64_t n, int64_t M) {
+    Layout L;
+    size_t off = 0;
+    const long long nchunks = ceil_div(M, kChunk);
+    L.wl_cap = wl_capacity(M);
+    L.stats = off;    off = align_up(off + sizeof(ecl_mst_stats), 256);
+    L.internal = off; off = align_up(off + sizeof(Internal), 256);
+    L.trace = off;    off = align_up(off + sizeof(long long) * kTraceSlots * kMaxGrid, 256);
+    L.rowstart = off; off = align_up(off + sizeof(int) * (size_t)(nchunks + 1), 256);
+    L.region = off;   off = align_up(off + sizeof(int4) * (size_t)kMaxPopWarps, 256);
+    L.giant = off;    off = align_up(off + sizeof(unsigned) * (size_t)((n + 31) / 32 + 1), 256);
+    L.key = off;      off = align_up(off + sizeof(long long) * (size_t)n, 256);
+    L.parent = off;   off = align_up(off + sizeof(int) * (size_t)n, 256);
+    L.wl0 = off;      off = align_up(off + sizeof(int4) * (size_t)L.wl_cap, 256);
+    L.wl1 = off;      off = align_up(off + sizeof(int4) * (size_t)L.wl_cap, 256);
+    L.total = off;
+    return L;
+}
+
+struct Params {
+    int n;
+    long long M;
+    long long nchunks;                // ceil(M / kChunk)
+    int G;                            // k_rounds CTAs = arenas
+    long long cap;                    // tuples per arena (k_rounds worklists)
+    int W;                            // populate warps = regions of wl0
+    long long rcap;                   // tuples per region
+    const long long* __restrict__ nindex;
+    const int* __restrict__ nlist;
+    const int* __restrict__ eweight;
+    unsigned char* in_mst;
+    long long* total_out;
+    ecl_mst_stats* st;
+    Internal* in;
+    long long* trace;                 // [kTraceSlots][kMaxGrid] or null
+    int* rowstart;                    // row of CSR entry c*kChunk, per chunk
+    int4* region;                     // per populate warp: {tuples, canonical, heavy, 0}
+    unsigned* giant_bits;             // bit v: v is in the largest set after phase 1 (or null)
+    long long* key;
+    int* parent;
+    int4* wl0;
+    int4* wl1;
+    unsigned long long seed;
+    int filter_mode;
+    int threshold_mode;
+    int threshold_value;
+    int samples;
+    int halving;
+    int guards;                       // -1 auto, 0 off, 1 on
+    int flatten;
+    // edge sharding (distributed path; single GPU: shard 0 of 1)
+    int shard;                        // global shard id
+    int nshards;                      // total shards
+    long long nlocal;                 // chunks of this shard: shard, shard + nshards, ...
+    int zero_mst;                     // populate phase 1 zeroes its chunks of in_mst
+    int* acnt;                        // per arena tuple count (distributed pass A)
+    int* tgt;                         // per vertex hook target (distributed rep pass)
+    long long* const* keys_all;       // virtual shards: every shard's key array
+    int nkeys;
+};
+
+__device__ __forceinline__ DS ds_of(const Params& P) {
+    DS D;
+    D.parent = P.parent;
+    D.key = P.key;
+    return D;
+}
+
+__device__ __forceinline__ void stamp(const Params& P, int slot) {
+    if (blockIdx.x == 0 && threadIdx.x == 0 && slot < kTraceSlots)
+        P.st->t_ns[slot] = (long long)globaltimer_ns();
+}
+
+// per-CTA end of a stage (diagnostics; P.trace is null unless opts.trace)
+__device__ __forceinline__ void trace_cta(const Params& P, int slot) {
+    if (P.trace && slot < kTraceSlots) {
+        __syncthreads();
+        if (threadIdx.x == 0) P.trace[(long long)slot * kMaxGrid + blockIdx.x] = (long long)globaltimer_ns();
+    }
+}
+
+// phase 2 runs iff filtering is on and phase 1 deferred at least one edge
+// (read-only within the kernels that ask: one L1 line per SM, not one L2
+// slice hammered by every warp of the grid)
+__device__ __forceinline__ bool phase2_needed(const Params& P) {
+    return __ldg(&P.st->filtered) != 0 && __ldg(&P.st->heavy_edges) != 0;
+}
+
+}  // namespace eclmst

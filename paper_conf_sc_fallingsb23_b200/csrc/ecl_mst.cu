@@ -30,12 +30,7 @@
 //                 (one load each after flattening), intra-set edges filtered.
 //   k_rounds      phase 2 rounds (exits at once when there is no phase 2).
 //   k_finalize    total weight / status -> caller's output.
-#include <cooperative_groups.h>
-#include <cuda_runtime.h>
-
-#include <climits>
 #include <cstdarg>
-#include <cstdint>
 #include <cstdio>
 #include <cstring>
 #include <dlfcn.h>
@@ -45,944 +40,12 @@
 #include <string>
 #include <vector>
 
-#include "device.cuh"
-#include "ecl_mst.h"
-
-namespace cg = cooperative_groups;
+#include "common.cuh"
+#include "populate.cuh"
+#include "rounds.cuh"
+#include "dist_kernels.cuh"
 
 namespace eclmst {
-
-constexpr int kMaxGrid = 4096;                 // CTAs of k_rounds (= arenas), upper bound
-constexpr int kPopWarps = 8;                   // warps per k_populate CTA (one chunk each)
-constexpr int kPopBlock = 32 * kPopWarps;
-constexpr int kMaxPopWarps = 65536;            // populate warps (= worklist regions), upper bound
-constexpr int kMaxRegionsPerCta = 256;         // regions a k_rounds CTA starts from
-constexpr int kTraceSlots = 2 * ECL_MST_MAX_ROUNDS + 4;
-constexpr int kMaxSamples = 4096;              // threshold sample size cap
-static_assert(kMaxGrid == ECL_MST_TRACE_CTAS, "trace layout");
-
-struct Internal {
-    unsigned long long reps;           // distributed path: sets with a finite key this round
-    unsigned int done;                 // unused ticket
-    int g_cur;                         // first global round of the running phase
-    int g_end;                         // last global round of the finished phase
-    int giant;                         // root of the largest set after phase 1 (-1: none)
-    int pad0;
-};
-
-struct Layout {
-    size_t stats, internal, trace, rowstart, region, giant, key, parent, wl0, wl1, total;
-    long long wl_cap;                  // tuples per worklist buffer
-};
-
-static inline size_t align_up(size_t x, size_t a) { return (x + a - 1) / a * a; }
-
-static inline long long ceil_div(long long a, long long b) { return (a + b - 1) / b; }
-
-// worklist tuples needed for W populate regions of ceil(nchunks/W)*kChunk
-// tuples, for any W <= min(kMaxPopWarps, nchunks)
-static inline long long wl_capacity(long long M) {
-    const long long nchunks = ceil_div(M, kChunk);
-    const long long wmax = nchunks < kMaxPopWarps ? nchunks : kMaxPopWarps;
-    return (nchunks + wmax) * (long long)kChunk;
-}
-
-static inline Layout layout_for(int64_t n, int64_t M) {
-    Layout L;
-    size_t off = 0;
-    const long long nchunks = ceil_div(M, kChunk);
-    L.wl_cap = wl_capacity(M);
-    L.stats = off;    off = align_up(off + sizeof(ecl_mst_stats), 256);
-    L.internal = off; off = align_up(off + sizeof(Internal), 256);
-    L.trace = off;    off = align_up(off + sizeof(long long) * kTraceSlots * kMaxGrid, 256);
-    L.rowstart = off; off = align_up(off + sizeof(int) * (size_t)(nchunks + 1), 256);
-    L.region = off;   off = align_up(off + sizeof(int4) * (size_t)kMaxPopWarps, 256);
-    L.giant = off;    off = align_up(off + sizeof(unsigned) * (size_t)((n + 31) / 32 + 1), 256);
-    L.key = off;      off = align_up(off + sizeof(long long) * (size_t)n, 256);
-    L.parent = off;   off = align_up(off + sizeof(int) * (size_t)n, 256);
-    L.wl0 = off;      off = align_up(off + sizeof(int4) * (size_t)L.wl_cap, 256);
-    L.wl1 = off;      off = align_up(off + sizeof(int4) * (size_t)L.wl_cap, 256);
-    L.total = off;
-    return L;
-}
-
-struct Params {
-    int n;
-    long long M;
-    long long nchunks;                // ceil(M / kChunk)
-    int G;                            // k_rounds CTAs = arenas
-    long long cap;                    // tuples per arena (k_rounds worklists)
-    int W;                            // populate warps = regions of wl0
-    long long rcap;                   // tuples per region
-    const long long* __restrict__ nindex;
-    const int* __restrict__ nlist;
-    const int* __restrict__ eweight;
-    unsigned char* in_mst;
-    long long* total_out;
-    ecl_mst_stats* st;
-    Internal* in;
-    long long* trace;                 // [kTraceSlots][kMaxGrid] or null
-    int* rowstart;                    // row of CSR entry c*kChunk, per chunk
-    int4* region;                     // per populate warp: {tuples, canonical, heavy, 0}
-    unsigned* giant_bits;             // bit v: v is in the largest set after phase 1 (or null)
-    long long* key;
-    int* parent;
-    int4* wl0;
-    int4* wl1;
-    unsigned long long seed;
-    int filter_mode;
-    int threshold_mode;
-    int threshold_value;
-    int samples;
-    int halving;
-    int guards;                       // -1 auto, 0 off, 1 on
-    int flatten;
-    // edge sharding (distributed path; single GPU: shard 0 of 1)
-    int shard;                        // global shard id
-    int nshards;                      // total shards
-    long long nlocal;                 // chunks of this shard: shard, shard + nshards, ...
-    int zero_mst;                     // populate phase 1 zeroes its chunks of in_mst
-    int* acnt;                        // per arena tuple count (distributed pass A)
-    int* tgt;                         // per vertex hook target (distributed rep pass)
-    long long* const* keys_all;       // virtual shards: every shard's key array
-    int nkeys;
-};
-
-__device__ __forceinline__ DS ds_of(const Params& P) {
-    DS D;
-    D.parent = P.parent;
-    D.key = P.key;
-    return D;
-}
-
-__device__ __forceinline__ void stamp(const Params& P, int slot) {
-    if (blockIdx.x == 0 && threadIdx.x == 0 && slot < kTraceSlots)
-        P.st->t_ns[slot] = (long long)globaltimer_ns();
-}
-
-// per-CTA end of a stage (diagnostics; P.trace is null unless opts.trace)
-__device__ __forceinline__ void trace_cta(const Params& P, int slot) {
-    if (P.trace && slot < kTraceSlots) {
-        __syncthreads();
-        if (threadIdx.x == 0) P.trace[(long long)slot * kMaxGrid + blockIdx.x] = (long long)globaltimer_ns();
-    }
-}
-
-// phase 2 runs iff filtering is on and phase 1 deferred at least one edge
-// (read-only within the kernels that ask: one L1 line per SM, not one L2
-// slice hammered by every warp of the grid)
-__device__ __forceinline__ bool phase2_needed(const Params& P) {
-    return __ldg(&P.st->filtered) != 0 && __ldg(&P.st->heavy_edges) != 0;
-}
-
-// ---------------------------------------------------------------------------
-// k_init: Alg. 1 + chunk start rows + threshold
-// ---------------------------------------------------------------------------
-__global__ void __launch_bounds__(256) k_init(Params P) {
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const long long stride = (long long)gridDim.x * blockDim.x;
-    const long long i0 = (long long)blockIdx.x * blockDim.x + tid;
-    bool err = false;
-    for (long long v = i0; v < P.n; v += stride) {
-        P.parent[v] = (int)v;                       // every vertex its own set
-        if (P.keys_all) {                           // no minimum edge recorded
-            for (int s2 = 0; s2 < P.nkeys; ++s2) P.keys_all[s2][v] = kInf;
-        } else {
-            P.key[v] = kInf;
-        }
-        // chunk starts inside row v: rowstart[c] = v for c*kChunk in [s, e)
-        const long long s = P.nindex[v], e = P.nindex[v + 1];
-        if (e < s) err = true;
-        for (long long c = (s + kChunk - 1) / kChunk; c * kChunk < e && c < P.nchunks; ++c) P.rowstart[c] = (int)v;
-    }
-    if (blockIdx.x == 0) {
-        ecl_mst_stats* st = P.st;   // zeroed by a memset node just before this kernel
-        __shared__ int s_w[kMaxSamples];
-        __shared__ int s_T;
-        // filter decision (readings Q5-Q7): estimate the
-        // weight of the c|V| lightest of the M entries (c = 4) from S random
-        // entries: T = the sample of rank floor(S * 4n / M)
-        const bool filtered = P.filter_mode < 0 ? (P.M >= 4LL * P.n) : (P.filter_mode != 0);
-        if (tid == 0) s_T = (filtered && P.threshold_mode == 1) ? P.threshold_value : INT_MAX;
-        if (filtered && P.threshold_mode == 0) {
-            const int S = P.samples;
-            for (int i = tid; i < S; i += blockDim.x) {
-                const unsigned long long h = splitmix64(P.seed * 0x100000001B3ull + (unsigned long long)i);
-                s_w[i] = P.eweight[(long long)(h % (unsigned long long)P.M)];
-            }
-            __syncthreads();
-            long long kpos = ((long long)S * 4LL * P.n) / P.M;
-            if (kpos > S - 1) kpos = S - 1;
-            for (int i = tid; i < S; i += blockDim.x) {
-                const int wi = s_w[i];
-                int rank = 0;
-                for (int t = 0; t < S; ++t) {
-                    const int wt = s_w[t];
-                    rank += (wt < wi) || (wt == wi && t < i);
-                }
-                if (rank == (int)kpos) s_T = wi;
-            }
-        }
-        __syncthreads();
-        if (tid == 0) {
-            st->t_ns[0] = (long long)globaltimer_ns();
-            st->filtered = filtered ? 1 : 0;
-            st->threshold = s_T;
-            st->grid = P.G;
-            st->block = kBlock;
-            st->phase2_round = -1;
-            if (P.nindex[0] != 0 || P.nindex[P.n] != P.M) err = true;
-            P.in->g_cur = 0;
-            P.in->g_end = 0;
-            P.in->done = 0;
-            P.in->giant = -1;
-        }
-    }
-    if (err) atomicExch(&P.st->status, ECL_MST_ERR_INPUT);
-}
-
-// ---------------------------------------------------------------------------
-// k_populate<PH>: one warp per 128-entry CSR chunk
-// ---------------------------------------------------------------------------
-template <int PH>
-#ifndef ECL_DEEP_PH1
-#define ECL_DEEP_PH1 0
-#endif
-#ifndef ECL_DEEP_PH2
-#define ECL_DEEP_PH2 1
-#endif
-#ifndef ECL_GIANT_MIN_N
-#define ECL_GIANT_MIN_N (32LL << 20)   // parent[] larger than ~half the L2
-#endif
-#ifndef ECL_POP_MINB
-#define ECL_POP_MINB 4
-#endif
-__global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) {
-    __shared__ int s_mark[kPopWarps][kChunk];
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    if (PH == 2 && !phase2_needed(P)) return;
-    if (blockIdx.x == 0 && threadIdx.x == 0) {
-        if (PH == 1) P.st->t_ns[1] = (long long)globaltimer_ns();   // init done
-        else P.st->t_ns[3] = (long long)globaltimer_ns();           // flatten done
-    }
-    const bool filtered = __ldg(&P.st->filtered) != 0;
-    const int T = __ldg(&P.st->threshold);
-    const bool guard = (P.guards > 0) || (P.guards < 0 && PH == 2);
-    const DS D = ds_of(P);
-    // warp w takes chunks w, w + W, ... (an even sample of the whole CSR, so
-    // every region -- and every k_rounds CTA -- gets the same mix even where
-    // the density of u < v entries drifts along the rows) and appends its
-    // tuples densely to its own region: no atomics, no CTA barrier.
-    const int w = blockIdx.x * kPopWarps + warp;
-    if (w >= P.W) return;
-    int4* const out = P.wl0 + (long long)w * P.rcap;
-    int cnt = 0, canon_cnt = 0, heavy_cnt = 0;
-    bool err = false;
-    const int p0 = lane * kItems;
-    // CSR entries of chunk c (lane owns entries p0 .. p0+3), streaming loads
-    auto load_entries = [&](long long c, int (&vv)[kItems], int (&ww)[kItems]) {
-        const long long c0 = c * kChunk;
-        const int len = (int)(min(c0 + (long long)kChunk, P.M) - c0);
-        if (p0 + kItems <= len) {
-            const int4 a = __ldcs(reinterpret_cast<const int4*>(P.nlist + c0 + p0));
-            const int4 b = __ldcs(reinterpret_cast<const int4*>(P.eweight + c0 + p0));
-            vv[0] = a.x; vv[1] = a.y; vv[2] = a.z; vv[3] = a.w;
-            ww[0] = b.x; ww[1] = b.y; ww[2] = b.z; ww[3] = b.w;
-        } else {
-#pragma unroll
-            for (int k = 0; k < kItems; ++k) {
-                const bool ok = p0 + k < len;
-                vv[k] = ok ? __ldcs(P.nlist + c0 + p0 + k) : -1;
-                ww[k] = ok ? __ldcs(P.eweight + c0 + p0 + k) : 0;
-            }
-        }
-    };
-    // software pipeline (edge sharding: this shard owns chunks shard,
-    // shard + nshards, ...; lc indexes them, c is the global chunk).  While
-    // chunk i is processed, chunk i+1's CSR entries and its first 64 row
-    // starts, and chunk i+2's row bracket, are in flight; at the end of
-    // chunk i the phase-2 membership bits of chunk i+1's far ends are
-    // requested (their entries have arrived by then).
-    const int giant = (PH == 2 && P.flatten && P.giant_bits) ? __ldg(&P.in->giant) : -1;
-    // deep: also prefetch the next chunk's row starts (phase 2, where the
-    // bitmap / parent loads already lengthen each chunk's chain)
-    constexpr bool deep = PH == 1 ? ECL_DEEP_PH1 : ECL_DEEP_PH2;
-    auto bracket = [&](long long lc, int& r0, int& rl) {
-        const long long c = P.shard + lc * P.nshards;
-        r0 = __ldg(P.rowstart + c);
-        rl = (c + 1 < P.nchunks) ? __ldg(P.rowstart + c + 1) : P.n - 1;
-    };
-    auto starts = [&](int r0, int rl, long long& sa, long long& sz) {
-        const int ra = r0 + 1 + lane, rz = r0 + 33 + lane;
-        sa = ra <= rl ? __ldg(P.nindex + ra) : LLONG_MAX;
-        sz = rz <= rl ? __ldg(P.nindex + rz) : LLONG_MAX;
-    };
-    auto vbits = [&](const int (&vv)[kItems]) {
-        unsigned b = 0;
-        if (PH == 2 && giant >= 0) {
-#pragma unroll
-            for (int k = 0; k < kItems; ++k)
-                if ((unsigned)vv[k] < (unsigned)P.n)
-                    b |= ((__ldg(P.giant_bits + (vv[k] >> 5)) >> (vv[k] & 31)) & 1u) << k;
-        }
-        return b;
-    };
-    int nr0 = 0, nrl = 0, n2r0 = 0, n2rl = 0, nv[kItems], nw[kItems];
-    long long nsa = LLONG_MAX, nsz = LLONG_MAX;
-    unsigned nvb = 0;
-    if (w < P.nlocal) {
-        bracket(w, nr0, nrl);
-        load_entries(P.shard + (long long)w * P.nshards, nv, nw);
-        if (deep) {
-            starts(nr0, nrl, nsa, nsz);
-            if (w + P.W < P.nlocal) bracket(w + P.W, n2r0, n2rl);
-        }
-        nvb = vbits(nv);
-    }
-    for (long long lc = w; lc < P.nlocal; lc += P.W) {
-    const long long c = P.shard + lc * P.nshards;
-    bool keep[kItems];
-    int4 t[kItems];
-#pragma unroll
-    for (int k = 0; k < kItems; ++k) keep[k] = false;
-    {
-        const long long c0 = c * kChunk;
-        const long long c1 = min(c0 + (long long)kChunk, P.M);
-        const int len = (int)(c1 - c0);
-        // rows of this chunk: r0 = row of entry c0; rows r0+1 .. r_last start inside
-        const int r0 = nr0, r_last = nrl;
-        const long long sa = nsa, sz = nsz;
-        const unsigned vb = nvb;
-        int vv[kItems], ww[kItems];
-#pragma unroll
-        for (int k = 0; k < kItems; ++k) {
-            vv[k] = nv[k];
-            ww[k] = nw[k];
-        }
-        const long long lcn = lc + P.W;
-        if (lcn < P.nlocal) {
-            load_entries(P.shard + lcn * P.nshards, nv, nw);
-            if (deep) {
-                nr0 = n2r0;
-                nrl = n2rl;
-                starts(nr0, nrl, nsa, nsz);
-                if (lcn + P.W < P.nlocal) bracket(lcn + P.W, n2r0, n2rl);
-            } else {
-                bracket(lcn, nr0, nrl);
-            }
-        }
-        int* mark = s_mark[warp];
-#pragma unroll
-        for (int i = lane; i < kChunk; i += 32) mark[i] = -1;
-        __syncwarp();
-        if (deep) {   // the first 64 row starts arrived with the prefetch
-            const int ra = r0 + 1 + lane, rz = r0 + 33 + lane;
-            if (sa >= c0 && sa < c1) atomicMax(&mark[sa - c0], ra);
-            else if (sa < c0) err = true;
-            if (sz >= c0 && sz < c1) atomicMax(&mark[sz - c0], rz);
-            else if (sz < c0) err = true;
-        }
-        for (int rb = r0 + (deep ? 65 : 1); rb <= r_last; rb += 64) {   // (further) row starts
-            const int ra = rb + lane, rz = rb + 32 + lane;
-            const long long ta = ra <= r_last ? __ldg(P.nindex + ra) : LLONG_MAX;
-            const long long tz = rz <= r_last ? __ldg(P.nindex + rz) : LLONG_MAX;
-            if (ta >= c0 && ta < c1) atomicMax(&mark[ta - c0], ra);
-            else if (ta < c0) err = true;
-            if (tz >= c0 && tz < c1) atomicMax(&mark[tz - c0], rz);
-            else if (tz < c0) err = true;
-        }
-        __syncwarp();
-        int row[kItems];
-#pragma unroll
-        for (int k = 0; k < kItems; ++k) row[k] = mark[p0 + k];
-        // inclusive max-scan over the warp's 128 positions
-#pragma unroll
-        for (int k = 1; k < kItems; ++k) row[k] = max(row[k], row[k - 1]);
-        int incl = row[kItems - 1];
-#pragma unroll
-        for (int o = 1; o < 32; o <<= 1) {
-            const int y = __shfl_up_sync(kFull, incl, o);
-            if (lane >= o) incl = max(incl, y);
-        }
-        int excl = __shfl_up_sync(kFull, incl, 1);
-        if (lane == 0) excl = r0;                 // position 0 belongs to row r0
-#pragma unroll
-        for (int k = 0; k < kItems; ++k) row[k] = max(row[k], max(excl, r0));
-
-        if (PH == 1 && P.zero_mst) {   // every in_mst byte is written once, here (Alg. 1 "not in MST")
-            if (p0 + kItems <= len) {
-                __stcs(reinterpret_cast<unsigned*>(P.in_mst + c0 + p0), 0u);
-            } else {
-#pragma unroll
-                for (int k = 0; k < kItems; ++k)
-                    if (p0 + k < len) P.in_mst[c0 + p0 + k] = 0;
-            }
-        }
-        bool cand[kItems];
-#pragma unroll
-        for (int k = 0; k < kItems; ++k) {
-            const bool valid = p0 + k < len;
-            const bool in_range = (unsigned)vv[k] < (unsigned)P.n;
-            if (valid && !in_range) err = true;
-            const bool canon = valid && in_range && row[k] < vv[k];   // L4: one direction only
-            const bool heavy = filtered && ww[k] >= T;                // L6 threshold condition
-            if (PH == 1) {
-                canon_cnt += canon;
-                heavy_cnt += (canon && heavy);
-                cand[k] = canon && !heavy;
-            } else {
-                cand[k] = canon && heavy;
-            }
-        }
-        int pk[kItems], qk[kItems];
-#pragma unroll
-        for (int k = 0; k < kItems; ++k) {
-            pk[k] = row[k];
-            qk[k] = vv[k];
-        }
-        if (PH == 2) {   // set(v), set(n): one load each after k_flatten
-#pragma unroll
-            for (int k = 0; k < kItems; ++k) {
-                if (cand[k] && giant >= 0 && ((vb >> k) & 1u) &&
-                    ((__ldg(P.giant_bits + (row[k] >> 5)) >> (row[k] & 31)) & 1)) {
-                    pk[k] = qk[k] = giant;                    // both ends in the largest set: filtered
-                } else if (cand[k]) {
-                    pk[k] = (k > 0 && cand[k - 1] && row[k] == row[k - 1]) ? -1 : __ldca(D.par(row[k]));
-                    qk[k] = __ldca(D.par(vv[k]));
-                }
-            }
-#pragma unroll
-            for (int k = 1; k < kItems; ++k)
-                if (pk[k] == -1) pk[k] = pk[k - 1];
-            if (!P.flatten) {
-#pragma unroll
-                for (int k = 0; k < kItems; ++k) {
-                    if (cand[k]) {
-                        pk[k] = find_root(D, pk[k], P.halving != 0);
-                        qk[k] = find_root(D, qk[k], P.halving != 0);
-                    }
-                }
-            }
-        }
-#pragma unroll
-        for (int k = 0; k < kItems; ++k) {
-            const long long j = c0 + p0 + k;
-            t[k] = make_int4(pk[k], qk[k], ww[k], (int)(unsigned)j);
-            keep[k] = cand[k] && pk[k] != qk[k];                  // phase 2: the filter
-        }
-        // L19-21: the lane's entries come in row order, so merge equal p first
-        long long best = kInf;
-        int bp = -1;
-#pragma unroll
-        for (int k = 0; k < kItems; ++k) {
-            if (!keep[k]) continue;
-            const long long key = make_key(t[k].z, (unsigned)t[k].w);   // L19 val <- e_w : e_id
-            if (t[k].x != bp) {
-                if (bp >= 0) record_min(D.k(bp), best, guard);
-                bp = t[k].x;
-                best = key;
-            } else {
-                best = min(best, key);
-            }
-        }
-        if (bp >= 0) record_min(D.k(bp), best, guard);
-#pragma unroll
-        for (int k = 0; k < kItems; ++k)
-            if (keep[k]) record_min(D.k(t[k].y), make_key(t[k].z, (unsigned)t[k].w), guard);
-    }
-    if (PH == 2 && lc + P.W < P.nlocal) nvb = vbits(nv);   // next chunk's far-end bits
-    // L7: append the chunk's tuples to the warp's region
-    unsigned m[kItems];
-    int off[kItems];
-    int tot = 0;
-#pragma unroll
-    for (int i = 0; i < kItems; ++i) {
-        m[i] = __ballot_sync(kFull, keep[i]);
-        off[i] = tot;
-        tot += __popc(m[i]);
-    }
-    const unsigned lt = (1u << lane) - 1u;
-#pragma unroll
-    for (int i = 0; i < kItems; ++i)
-        if (keep[i]) __stcg(out + cnt + off[i] + __popc(m[i] & lt), t[i]);
-    cnt += tot;
-    }
-    if (err) atomicExch(&P.st->status, ECL_MST_ERR_INPUT);
-    if (PH == 1) {   // |E| and the deferred count of this warp's chunks
-        canon_cnt = warp_sum(canon_cnt);
-        heavy_cnt = warp_sum(heavy_cnt);
-    }
-    if (lane == 0) P.region[w] = make_int4(cnt, canon_cnt, heavy_cnt, 0);
-}
-
-// ---------------------------------------------------------------------------
-// k_flatten: parent[v] = find(v) before the phase-2 populate, so the phase-2
-// populate can use parent[x] as set(x) with one load.  Two launches: stage 1
-// compresses with path halving from every vertex (fast, but a halving store
-// of one thread can land after another thread's final root store and leave
-// a vertex one or two hops from its root); stage 2 finishes exactly with
-// owner-only pointer jumping (each slot written by the thread that owns it,
-// reads through L2 to see the others' progress), cheap on the short paths
-// stage 1 leaves.  Roots never change here.
-// ---------------------------------------------------------------------------
-template <int STAGE>
-__global__ void __launch_bounds__(256) k_flatten(Params P) {
-    if (!phase2_needed(P) || !P.flatten) return;
-    const long long stride = (long long)gridDim.x * blockDim.x;
-    const DS D = ds_of(P);
-    const int lane = threadIdx.x & 31;
-    const int giant = (STAGE == 2 && P.giant_bits) ? __ldcg(&P.in->giant) : -1;
-    // warps walk 32 consecutive vertices together (stage 2 ballots the bitmap)
-    for (long long base = (long long)blockIdx.x * blockDim.x + threadIdx.x - lane; base < P.n; base += stride) {
-        const long long v = base + lane;
-        const bool valid = v < P.n;
-        if (STAGE == 1) {
-            // fast, racy compression: path halving by everybody (ends close
-            // to, but not always exactly at, one hop)
-            if (valid) {
-                const int r = find_root(D, (int)v, true);
-                if (r != (int)v) *D.par(v) = r;
-            }
-        } else {
-            // exact: owner-only pointer jumping over the now-short paths
-            int p = valid ? __ldcg(D.par(v)) : -1;
-            while (valid) {
-                const int pp = __ldcg(D.par(p));
-                if (pp == p) break;
-                __stcg(D.par(v), pp);
-                p = pp;
-            }
-            if (P.giant_bits) {
-                const unsigned bits = __ballot_sync(kFull, valid && p == giant);
-                if (lane == 0) P.giant_bits[base >> 5] = bits;
-            }
-        }
-    }
-}
-
-// After phase 1 most vertices of a graph whose light edges percolate (C3-C5)
-// sit in ONE set.  Find its root by a majority vote over sampled vertices;
-// k_flatten<2> then writes a bitmap of its members, and the phase-2 populate
-// filters an edge with both ends in it from the bitmap (n/8 bytes, L2
-// resident) instead of two random parent loads.
-__global__ void __launch_bounds__(256) k_giant(Params P) {
-    __shared__ int s_r[1024];
-    if (!phase2_needed(P) || !P.flatten || !P.giant_bits) return;
-    const DS D = ds_of(P);
-    for (int i = threadIdx.x; i < 1024; i += blockDim.x) {
-        const long long v = (long long)(splitmix64(0x6A09E667F3BCC909ull + (unsigned long long)i) % (unsigned long long)P.n);
-        s_r[i] = find_root(D, (int)v, false);
-    }
-    __syncthreads();
-    if (threadIdx.x == 0) {
-        int cand = -1, votes = 0;                 // Boyer-Moore majority vote
-        for (int i = 0; i < 1024; ++i) {
-            if (votes == 0) { cand = s_r[i]; votes = 1; }
-            else votes += (s_r[i] == cand) ? 1 : -1;
-        }
-        int cnt = 0;
-        for (int i = 0; i < 1024; ++i) cnt += s_r[i] == cand;
-        P.in->giant = cnt >= 256 ? cand : -1;     // worth a bitmap only if it holds >= 1/4
-    }
-}
-
-// ---------------------------------------------------------------------------
-// rounds: pass A / pass B over the CTA's arena
-// ---------------------------------------------------------------------------
-
-// A CTA's worklist as a sequence of 128-tuple chunks.  Right after populate
-// it is the CTA's share of the populate regions (regions b, b+G, ..., each a
-// dense run of region[w].x tuples; chunk j maps to a region by a binary
-// search over the shared prefix s_pre) -- RegionSrc; after a pass A it is one
-// compact run of cnt tuples -- CompactSrc.  Two types, so each pass is
-// compiled once per mode and carries only the registers that mode needs.
-struct CompactSrc {
-    const int4* base;
-    int cnt;
-    int nloc;
-    __device__ __forceinline__ const int4* get(const Params&, int j, int& count) const {
-        count = min(kChunk, cnt - j * kChunk);
-        return base + (long long)j * kChunk;
-    }
-};
-
-struct RegionSrc {
-    const int* s_pre;   // shared memory: chunk prefix per region (nreg + 1)
-    const int* s_rcnt;  // shared memory: tuples per region
-    int nreg;
-    int nloc;
-    int first_w;
-    __device__ __forceinline__ const int4* get(const Params& P, int j, int& count) const {
-        int lo = 0, hi = nreg;
-        while (hi - lo > 1) {
-            const int mid = (lo + hi) >> 1;
-            if (s_pre[mid] <= j) lo = mid;
-            else hi = mid;
-        }
-        const int off = j - s_pre[lo];
-        count = min(kChunk, s_rcnt[lo] - off * kChunk);
-        return P.wl0 + (long long)(first_w + lo * P.G) * P.rcap + (long long)off * kChunk;
-    }
-};
-
-__device__ __forceinline__ CompactSrc compact_src(const int4* base, int cnt) {
-    CompactSrc S;
-    S.base = base;
-    S.cnt = cnt;
-    S.nloc = (cnt + kChunk - 1) / kChunk;
-    return S;
-}
-
-// the populate output of CTA b: regions w = b, b + G, ...  Loads the region
-// counts into shared memory, builds the chunk prefix, and adds the kept,
-// canonical and deferred counts to the stats (phase 1 counters only if
-// count_phase1).  Every thread of the CTA must call it.
-__device__ __forceinline__ RegionSrc region_src(const Params& P, int b, int* s_pre, int* s_rcnt,
-                                                long long (*s_red)[kWarps], int64_t* live_slot,
-                                                bool count_phase1) {
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    RegionSrc R;
-    R.s_pre = s_pre;
-    R.s_rcnt = s_rcnt;
-    R.nreg = b < P.W ? (P.W - b + P.G - 1) / P.G : 0;
-    R.first_w = b;
-    long long canon = 0, heavy = 0;
-    for (int k = tid; k < R.nreg; k += kBlock) {
-        const int4 r = P.region[b + k * P.G];
-        s_rcnt[k] = r.x;
-        canon += r.y;
-        heavy += r.z;
-    }
-    canon = warp_sum(canon);
-    heavy = warp_sum(heavy);
-    if (lane == 0) {
-        s_red[1][warp] = canon;
-        s_red[2][warp] = heavy;
-    }
-    __syncthreads();
-    if (tid == 0) {
-        long long kept = 0;
-        int pre = 0;
-        for (int k = 0; k < R.nreg; ++k) {
-            s_pre[k] = pre;
-            pre += (s_rcnt[k] + kChunk - 1) / kChunk;
-            kept += s_rcnt[k];
-        }
-        s_pre[R.nreg] = pre;
-        canon = heavy = 0;
-        for (int w2 = 0; w2 < kWarps; ++w2) {
-            canon += s_red[1][w2];
-            heavy += s_red[2][w2];
-        }
-        if (kept) atomicAdd(reinterpret_cast<unsigned long long*>(live_slot), (unsigned long long)kept);
-        if (count_phase1) {
-            if (canon) atomicAdd(reinterpret_cast<unsigned long long*>(&P.st->canonical_edges), (unsigned long long)canon);
-            if (heavy) atomicAdd(reinterpret_cast<unsigned long long*>(&P.st->heavy_edges), (unsigned long long)heavy);
-        }
-    }
-    __syncthreads();
-    R.nloc = s_pre[R.nreg];
-    return R;
-}
-
-// L14-23 of one round over the CTA's worklist: S -> out (compact).
-template <class SRC>
-__device__ __forceinline__ void passA(const Params& P, const SRC& S, int4* __restrict__ out, int* s_out,
-                                      bool guard) {
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const bool halving = P.halving != 0;
-    const DS D = ds_of(P);
-    for (int k = warp; k < S.nloc; k += kWarps) {
-        int count;
-        const int4* __restrict__ in = S.get(P, k, count);
-        int4 t[kItems];
-        bool keep[kItems];
-#pragma unroll
-        for (int i = 0; i < kItems; ++i) {
-            const int idx = i * 32 + lane;
-            keep[i] = idx < count;
-            t[i] = keep[i] ? __ldcs(in + idx) : make_int4(0, 0, 0, 0);
-        }
-        int px[kItems], qx[kItems];
-#pragma unroll
-        for (int i = 0; i < kItems; ++i) {
-            if (keep[i]) {
-                px[i] = __ldca(D.par(t[i].x));
-                qx[i] = __ldca(D.par(t[i].y));
-            }
-        }
-#pragma unroll
-        for (int i = 0; i < kItems; ++i) {
-            if (keep[i]) {
-                const int p = find_from(D, t[i].x, px[i], halving);        // L15
-                const int q = find_from(D, t[i].y, qx[i], halving);        // L16
-                keep[i] = p != q;                                          // L17
-                t[i].x = p;                                                // L18: implicit
-                t[i].y = q;                                                //      path compression
-            }
-        }
-#pragma unroll
-        for (int i = 0; i < kItems; ++i) {
-            if (keep[i]) {
-                const long long key = make_key(t[i].z, (unsigned)t[i].w); // L19
-                record_min(D.k(t[i].x), key, guard);                      // L20
-                record_min(D.k(t[i].y), key, guard);                      // L21
-            }
-        }
-        warp_emit(t, keep, out, s_out);                                   // L18
-    }
-}
-
-// L27-31 (+ L34-37): check, join, mark over the CTA's worklist.
-template <class SRC>
-__device__ __forceinline__ void passB(const Params& P, const SRC& S, long long& wsum, long long& wcnt) {
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const DS D = ds_of(P);
-    for (int k = warp; k < S.nloc; k += kWarps) {
-        int count;
-        const int4* __restrict__ in = S.get(P, k, count);
-        int4 t[kItems];
-        bool ok[kItems];
-#pragma unroll
-        for (int i = 0; i < kItems; ++i) {
-            const int idx = i * 32 + lane;
-            ok[i] = idx < count;
-            t[i] = ok[i] ? __ldcg(in + idx) : make_int4(0, 0, 0, 0);
-        }
-        // Only the id half of each slot is compared: ids are unique per
-        // edge, so id equality is key equality (and inf's id half, 2^32-1,
-        // is never a valid id).  L1 is fine: K[p] only changes when p's own
-        // winner resets it.
-        unsigned kp[kItems], kq[kItems];
-#pragma unroll
-        for (int i = 0; i < kItems; ++i) {
-            if (ok[i]) {
-                kp[i] = __ldca(reinterpret_cast<const unsigned*>(D.k(t[i].x)));
-                kq[i] = __ldca(reinterpret_cast<const unsigned*>(D.k(t[i].y)));
-            }
-        }
-#pragma unroll
-        for (int i = 0; i < kItems; ++i) {
-            if (!ok[i]) continue;
-            const bool wp = kp[i] == (unsigned)t[i].w, wq = kq[i] == (unsigned)t[i].w;   // L29
-            if (wp || wq) {
-                const int p = t[i].x, q = t[i].y;
-                // L30 join: each set hooks along its own lightest edge;
-                // a mutual pair keeps the smaller representative as root.
-                if (wp && !(wq && p < q)) __stcg(D.par(p), q);
-                if (wq && !(wp && q < p)) __stcg(D.par(q), p);
-                if (wp) __stcg(D.k(p), kInf);                          // L35
-                if (wq) __stcg(D.k(q), kInf);                          // L36
-                P.in_mst[(unsigned)t[i].w] = 1;                        // L31
-                wsum += t[i].z;
-                wcnt += 1;
-            }
-        }
-    }
-}
-
-// guard policy for pass A.  "auto" guards when edges crowd onto few
-// sets -- each set with a live edge produced exactly one winner last round
-// (mutual pairs: one for two sets), so live / winners estimates the number of
-// edges per set that would atomicMin the same slot -- or when the key array
-// is far larger than L2 (n >= 2^25: every unguarded atomic on a random slot
-// is a DRAM read-modify-write, a guard miss only a read).  Measured: C5 and
-// C4 gain, C2/C3 lose with guards in every round.
-__device__ __forceinline__ bool use_guard(const Params& P, long long live, long long winners) {
-    if (P.guards >= 0) return P.guards != 0;
-    return live > 8 * winners || P.n >= (1 << 25);
-}
-
-template <int PH>
-__global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
-    cg::grid_group grid = cg::this_grid();
-    __shared__ int s_out;
-    __shared__ long long s_red[3][kWarps];
-    __shared__ int s_pre[kMaxRegionsPerCta + 1];
-    __shared__ int s_rcnt[kMaxRegionsPerCta];
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const bool b0 = blockIdx.x == 0;
-    ecl_mst_stats* st = P.st;
-    if (PH == 2 && !phase2_needed(P)) return;
-    int g = (PH == 1) ? 0 : __ldcg(&P.in->g_end) + 1;
-    if (g >= ECL_MST_MAX_ROUNDS) {
-        if (b0 && tid == 0) atomicExch(&st->status, ECL_MST_ERR_INPUT);
-        return;
-    }
-    stamp(P, 4 + 2 * g);                      // populate done
-    const int b = blockIdx.x;
-    int4* wl[2] = {P.wl0 + (long long)b * P.cap, P.wl1 + (long long)b * P.cap};
-    // the populate output of this CTA: regions w = b, b + G, ... (region mode)
-    const RegionSrc R = region_src(P, b, s_pre, s_rcnt, s_red, &st->live[g], PH == 1);
-    if (b0 && tid == 0 && PH == 2) st->phase2_round = g;
-    trace_cta(P, 4 + 2 * g);
-    grid.sync();
-    long long wsum = 0, wcnt = 0;
-    int cur = 0;
-    bool overflow = false;
-    long long L = __ldcg(&st->live[g]);
-    CompactSrc C = compact_src(wl[0], 0);
-    // one round: pass B over S, then pass A from S into the other worklist
-    auto round = [&](const auto& S) {
-        const long long w0 = wcnt;
-        passB(P, S, wsum, wcnt);
-        const long long d = warp_sum(wcnt - w0);
-        if (lane == 0 && d) atomicAdd(reinterpret_cast<unsigned long long*>(&st->winners[g]), (unsigned long long)d);
-        if (tid == 0) s_out = 0;
-        trace_cta(P, 5 + 2 * g);
-        grid.sync();
-        stamp(P, 5 + 2 * g);
-        if (g + 1 >= ECL_MST_MAX_ROUNDS) {
-            overflow = true;
-            return false;
-        }
-        const bool guard = use_guard(P, L, __ldcg(&st->winners[g]));
-        ++g;
-        passA(P, S, wl[cur ^ 1], &s_out, guard);
-        cur ^= 1;
-        __syncthreads();
-        C = compact_src(wl[cur], s_out);
-        if (tid == 0 && C.cnt) atomicAdd(reinterpret_cast<unsigned long long*>(&st->live[g]), (unsigned long long)C.cnt);
-        trace_cta(P, 4 + 2 * g);
-        grid.sync();
-        stamp(P, 4 + 2 * g);
-        L = __ldcg(&st->live[g]);
-        return true;
-    };
-    if (L > 0 && round(R))
-        while (L > 0 && round(C)) {
-        }
-    const long long s = warp_sum(wsum), c = warp_sum(wcnt);
-    if (lane == 0) {
-        if (s) atomicAdd(reinterpret_cast<unsigned long long*>(&st->total_weight), (unsigned long long)s);
-        if (c) atomicAdd(reinterpret_cast<unsigned long long*>(&st->msf_edges), (unsigned long long)c);
-    }
-    if (b0 && tid == 0) {
-        P.in->g_end = g;
-        st->rounds = g + 1;
-        if (overflow) atomicExch(&st->status, ECL_MST_ERR_INPUT);
-    }
-}
-
-__global__ void k_finalize(Params P) {
-    if (threadIdx.x == 0) {
-        ecl_mst_stats* st = P.st;
-        st->t_ns[2] = (long long)globaltimer_ns();
-        const int status = *reinterpret_cast<volatile int*>(&st->status);
-        *P.total_out = status ? LLONG_MIN : *reinterpret_cast<volatile long long*>(&st->total_weight);
-    }
-}
-
-
-// ---------------------------------------------------------------------------
-// Distributed (edge-sharded) MSF -- SURVEY §8(e).  Every rank holds the full
-// CSR, a replicated union-find and a full key array; it owns the CSR chunks
-// c = shard, shard + P, ... and the tuples they produce.  Per round:
-//   allreduce(key, min) over the ranks  ->  every rank knows each set's
-//   lightest edge;  rep-centric pass B, identical on every rank (each set
-//   with a finite key hooks along its edge, looked up by id in the CSR);
-//   local pass A over the rank's own tuples.
-// ---------------------------------------------------------------------------
-
-// row of CSR entry j: binary search inside the rows of j's chunk
-__device__ __forceinline__ int row_of_entry(const Params& P, long long j) {
-    const long long c = j / kChunk;
-    int lo = __ldg(P.rowstart + c);
-    int hi = (c + 1 < P.nchunks) ? __ldg(P.rowstart + c + 1) : P.n - 1;
-    while (lo < hi) {   // largest r in [lo, hi] with nindex[r] <= j
-        const int mid = lo + ((hi - lo + 1) >> 1);
-        if (__ldg(P.nindex + mid) <= j) lo = mid;
-        else hi = mid - 1;
-    }
-    return lo;
-}
-
-// virtual shards on one GPU: the "allreduce" is an elementwise min over the
-// shards' key arrays, written back to every copy (as NCCL would)
-__global__ void __launch_bounds__(256) k_vreduce(Params P) {
-    const long long stride = (long long)gridDim.x * blockDim.x;
-    for (long long v = (long long)blockIdx.x * blockDim.x + threadIdx.x; v < P.n; v += stride) {
-        long long m = kInf;
-        for (int s2 = 0; s2 < P.nkeys; ++s2) m = min(m, P.keys_all[s2][v]);
-        for (int s2 = 0; s2 < P.nkeys; ++s2) P.keys_all[s2][v] = m;
-    }
-}
-
-// rep pass 1: for every set x with a finite (reduced) key, the other end's set
-// q of its lightest edge, and whether that edge is q's lightest too (mutual)
-__global__ void __launch_bounds__(256) k_dist_reps1(Params P) {
-    const long long stride = (long long)gridDim.x * blockDim.x;
-    unsigned long long found = 0;
-    for (long long x = (long long)blockIdx.x * blockDim.x + threadIdx.x; x < P.n; x += stride) {
-        const long long kx = P.key[x];   // distributed path: own arrays (stride 1)
-        if (kx == kInf) continue;
-        ++found;
-        const unsigned j = (unsigned)(kx & 0xffffffffll);
-        const int u = row_of_entry(P, (long long)j);
-        const int v = __ldg(P.nlist + j);
-        const DS D = ds_of(P);
-        const int pu = find_root(D, u, false), pv = find_root(D, v, false);
-        const int q = (pu == (int)x) ? pv : pu;
-        const bool mutual = P.key[q] == kx;
-        P.tgt[x] = q | (mutual ? (int)0x80000000 : 0);
-    }
-    found = warp_sum(found);
-    if ((threadIdx.x & 31) == 0 && found) atomicAdd(reinterpret_cast<unsigned long long*>(&P.in->reps), found);
-}
-
-// rep pass 2 (L30-31, L34-37): hook, mark, sum, reset -- the same rule as the
-// tuple-centric pass B, so the partition after each round is the same
-__global__ void __launch_bounds__(256) k_dist_reps2(Params P, int g) {
-    const long long stride = (long long)gridDim.x * blockDim.x;
-    long long wsum = 0, wcnt = 0;
-    for (long long x = (long long)blockIdx.x * blockDim.x + threadIdx.x; x < P.n; x += stride) {
-        const long long kx = P.key[x];
-        if (kx == kInf) continue;
-        const int t = P.tgt[x];
-        const int q = t & 0x7fffffff;
-        const bool mutual = t < 0;
-        if (!mutual || (int)x > q) P.parent[x] = q;
-        if (!mutual || (int)x < q) {
-            P.in_mst[(unsigned)(kx & 0xffffffffll)] = 1;
-            wsum += (int)(kx >> 32);
-            wcnt += 1;
-        }
-        for (int s2 = 0; s2 < P.nkeys; ++s2) P.keys_all[s2][x] = kInf;
-    }
-    wsum = warp_sum(wsum);
-    wcnt = warp_sum(wcnt);
-    if ((threadIdx.x & 31) == 0 && wcnt) {
-        atomicAdd(reinterpret_cast<unsigned long long*>(&P.st->total_weight), (unsigned long long)wsum);
-        atomicAdd(reinterpret_cast<unsigned long long*>(&P.st->msf_edges), (unsigned long long)wcnt);
-        atomicAdd(reinterpret_cast<unsigned long long*>(&P.st->winners[g]), (unsigned long long)wcnt);
-    }
-}
-
-// local pass A of shard P.shard: CTA b reads arena b (FIRST: its populate
-// regions), compacts the survivors into the other worklist
-template <bool FIRST>
-__global__ void __launch_bounds__(kBlock, 2) k_dist_passA(Params P, int g, int cur) {
-    __shared__ int s_out;
-    __shared__ long long s_red[3][kWarps];
-    __shared__ int s_pre[kMaxRegionsPerCta + 1];
-    __shared__ int s_rcnt[kMaxRegionsPerCta];
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    const int b = blockIdx.x;
-    int4* wl[2] = {P.wl0 + (long long)b * P.cap, P.wl1 + (long long)b * P.cap};
-    if (tid == 0) s_out = 0;
-    if (FIRST) {
-        const RegionSrc R = region_src(P, b, s_pre, s_rcnt, s_red, &P.st->live[g - 1], g - 1 == 0);
-        passA(P, R, wl[cur ^ 1], &s_out, P.guards != 0);
-    } else {
-        __syncthreads();
-        passA(P, compact_src(wl[cur], P.acnt[b]), wl[cur ^ 1], &s_out, P.guards != 0);
-    }
-    __syncthreads();
-    if (tid == 0) {
-        P.acnt[b] = s_out;
-        if (s_out) atomicAdd(reinterpret_cast<unsigned long long*>(&P.st->live[g]), (unsigned long long)s_out);
-    }
-}
 
 // ---------------------------------------------------------------------------
 // host side

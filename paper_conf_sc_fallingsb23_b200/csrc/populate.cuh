@@ -1,0 +1,350 @@
+// populate.cuh -- k_init (Alg. 1, chunk start rows, threshold sample) and
+// k_populate (Alg. 2 L1-11 fused with round 0 of L14-21; phase 2 with the
+// cycle filter).
+#pragma once
+
+#include "common.cuh"
+
+namespace eclmst {
+
+// ---------------------------------------------------------------------------
+// k_init: Alg. 1 + chunk start rows + threshold
+// ---------------------------------------------------------------------------
+__global__ void __launch_bounds__(256) k_init(Params P) {
+    const int tid = threadIdx.x;
+    const long long stride = (long long)gridDim.x * blockDim.x;
+    const long long i0 = (long long)blockIdx.x * blockDim.x + tid;
+    bool err = false;
+    for (long long v = i0; v < P.n; v += stride) {
+        P.parent[v] = (int)v;                       // every vertex its own set
+        if (P.keys_all) {                           // no minimum edge recorded
+            for (int s2 = 0; s2 < P.nkeys; ++s2) P.keys_all[s2][v] = kInf;
+        } else {
+            P.key[v] = kInf;
+        }
+        // chunk starts inside row v: rowstart[c] = v for c*kChunk in [s, e)
+        const long long s = P.nindex[v], e = P.nindex[v + 1];
+        if (e < s) err = true;
+        for (long long c = (s + kChunk - 1) / kChunk; c * kChunk < e && c < P.nchunks; ++c) P.rowstart[c] = (int)v;
+    }
+    if (blockIdx.x == 0) {
+        ecl_mst_stats* st = P.st;   // zeroed by a memset node just before this kernel
+        __shared__ int s_w[kMaxSamples];
+        __shared__ int s_T;
+        // filter decision (readings Q5-Q7): estimate the
+        // weight of the c|V| lightest of the M entries (c = 4) from S random
+        // entries: T = the sample of rank floor(S * 4n / M)
+        const bool filtered = P.filter_mode < 0 ? (P.M >= 4LL * P.n) : (P.filter_mode != 0);
+        if (tid == 0) s_T = (filtered && P.threshold_mode == 1) ? P.threshold_value : INT_MAX;
+        if (filtered && P.threshold_mode == 0) {
+            const int S = P.samples;
+            for (int i = tid; i < S; i += blockDim.x) {
+                const unsigned long long h = splitmix64(P.seed * 0x100000001B3ull + (unsigned long long)i);
+                s_w[i] = P.eweight[(long long)(h % (unsigned long long)P.M)];
+            }
+            __syncthreads();
+            long long kpos = ((long long)S * 4LL * P.n) / P.M;
+            if (kpos > S - 1) kpos = S - 1;
+            for (int i = tid; i < S; i += blockDim.x) {
+                const int wi = s_w[i];
+                int rank = 0;
+                for (int t = 0; t < S; ++t) {
+                    const int wt = s_w[t];
+                    rank += (wt < wi) || (wt == wi && t < i);
+                }
+                if (rank == (int)kpos) s_T = wi;
+            }
+        }
+        __syncthreads();
+        if (tid == 0) {
+            st->t_ns[0] = (long long)globaltimer_ns();
+            st->filtered = filtered ? 1 : 0;
+            st->threshold = s_T;
+            st->grid = P.G;
+            st->block = kBlock;
+            st->phase2_round = -1;
+            if (P.nindex[0] != 0 || P.nindex[P.n] != P.M) err = true;
+            P.in->g_cur = 0;
+            P.in->g_end = 0;
+            P.in->done = 0;
+            P.in->giant = -1;
+        }
+    }
+    if (err) atomicExch(&P.st->status, ECL_MST_ERR_INPUT);
+}
+
+// ---------------------------------------------------------------------------
+// k_populate<PH>: one warp per 128-entry CSR chunk
+// ---------------------------------------------------------------------------
+template <int PH>
+#ifndef ECL_DEEP_PH1
+#define ECL_DEEP_PH1 0
+#endif
+#ifndef ECL_DEEP_PH2
+#define ECL_DEEP_PH2 1
+#endif
+#ifndef ECL_GIANT_MIN_N
+#define ECL_GIANT_MIN_N (32LL << 20)   // parent[] larger than ~half the L2
+#endif
+#ifndef ECL_POP_MINB
+#define ECL_POP_MINB 4
+#endif
+__global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) {
+    __shared__ int s_mark[kPopWarps][kChunk];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    if (PH == 2 && !phase2_needed(P)) return;
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        if (PH == 1) P.st->t_ns[1] = (long long)globaltimer_ns();   // init done
+        else P.st->t_ns[3] = (long long)globaltimer_ns();           // flatten done
+    }
+    const bool filtered = __ldg(&P.st->filtered) != 0;
+    const int T = __ldg(&P.st->threshold);
+    const bool guard = (P.guards > 0) || (P.guards < 0 && PH == 2);
+    const DS D = ds_of(P);
+    // warp w takes chunks w, w + W, ... (an even sample of the whole CSR, so
+    // every region -- and every k_rounds CTA -- gets the same mix even where
+    // the density of u < v entries drifts along the rows) and appends its
+    // tuples densely to its own region: no atomics, no CTA barrier.
+    const int w = blockIdx.x * kPopWarps + warp;
+    if (w >= P.W) return;
+    int4* const out = P.wl0 + (long long)w * P.rcap;
+    int cnt = 0, canon_cnt = 0, heavy_cnt = 0;
+    bool err = false;
+    const int p0 = lane * kItems;
+    // CSR entries of chunk c (lane owns entries p0 .. p0+3), streaming loads
+    auto load_entries = [&](long long c, int (&vv)[kItems], int (&ww)[kItems]) {
+        const long long c0 = c * kChunk;
+        const int len = (int)(min(c0 + (long long)kChunk, P.M) - c0);
+        if (p0 + kItems <= len) {
+            const int4 a = __ldcs(reinterpret_cast<const int4*>(P.nlist + c0 + p0));
+            const int4 b = __ldcs(reinterpret_cast<const int4*>(P.eweight + c0 + p0));
+            vv[0] = a.x; vv[1] = a.y; vv[2] = a.z; vv[3] = a.w;
+            ww[0] = b.x; ww[1] = b.y; ww[2] = b.z; ww[3] = b.w;
+        } else {
+#pragma unroll
+            for (int k = 0; k < kItems; ++k) {
+                const bool ok = p0 + k < len;
+                vv[k] = ok ? __ldcs(P.nlist + c0 + p0 + k) : -1;
+                ww[k] = ok ? __ldcs(P.eweight + c0 + p0 + k) : 0;
+            }
+        }
+    };
+    // software pipeline (edge sharding: this shard owns chunks shard,
+    // shard + nshards, ...; lc indexes them, c is the global chunk).  While
+    // chunk i is processed, chunk i+1's CSR entries and its first 64 row
+    // starts, and chunk i+2's row bracket, are in flight; at the end of
+    // chunk i the phase-2 membership bits of chunk i+1's far ends are
+    // requested (their entries have arrived by then).
+    const int giant = (PH == 2 && P.flatten && P.giant_bits) ? __ldg(&P.in->giant) : -1;
+    // deep: also prefetch the next chunk's row starts (phase 2, where the
+    // bitmap / parent loads already lengthen each chunk's chain)
+    constexpr bool deep = PH == 1 ? ECL_DEEP_PH1 : ECL_DEEP_PH2;
+    auto bracket = [&](long long lc, int& r0, int& rl) {
+        const long long c = P.shard + lc * P.nshards;
+        r0 = __ldg(P.rowstart + c);
+        rl = (c + 1 < P.nchunks) ? __ldg(P.rowstart + c + 1) : P.n - 1;
+    };
+    auto starts = [&](int r0, int rl, long long& sa, long long& sz) {
+        const int ra = r0 + 1 + lane, rz = r0 + 33 + lane;
+        sa = ra <= rl ? __ldg(P.nindex + ra) : LLONG_MAX;
+        sz = rz <= rl ? __ldg(P.nindex + rz) : LLONG_MAX;
+    };
+    auto vbits = [&](const int (&vv)[kItems]) {
+        unsigned b = 0;
+        if (PH == 2 && giant >= 0) {
+#pragma unroll
+            for (int k = 0; k < kItems; ++k)
+                if ((unsigned)vv[k] < (unsigned)P.n)
+                    b |= ((__ldg(P.giant_bits + (vv[k] >> 5)) >> (vv[k] & 31)) & 1u) << k;
+        }
+        return b;
+    };
+    int nr0 = 0, nrl = 0, n2r0 = 0, n2rl = 0, nv[kItems], nw[kItems];
+    long long nsa = LLONG_MAX, nsz = LLONG_MAX;
+    unsigned nvb = 0;
+    if (w < P.nlocal) {
+        bracket(w, nr0, nrl);
+        load_entries(P.shard + (long long)w * P.nshards, nv, nw);
+        if (deep) {
+            starts(nr0, nrl, nsa, nsz);
+            if (w + P.W < P.nlocal) bracket(w + P.W, n2r0, n2rl);
+        }
+        nvb = vbits(nv);
+    }
+    for (long long lc = w; lc < P.nlocal; lc += P.W) {
+    const long long c = P.shard + lc * P.nshards;
+    bool keep[kItems];
+    int4 t[kItems];
+#pragma unroll
+    for (int k = 0; k < kItems; ++k) keep[k] = false;
+    {
+        const long long c0 = c * kChunk;
+        const long long c1 = min(c0 + (long long)kChunk, P.M);
+        const int len = (int)(c1 - c0);
+        // rows of this chunk: r0 = row of entry c0; rows r0+1 .. r_last start inside
+        const int r0 = nr0, r_last = nrl;
+        const long long sa = nsa, sz = nsz;
+        const unsigned vb = nvb;
+        int vv[kItems], ww[kItems];
+#pragma unroll
+        for (int k = 0; k < kItems; ++k) {
+            vv[k] = nv[k];
+            ww[k] = nw[k];
+        }
+        const long long lcn = lc + P.W;
+        if (lcn < P.nlocal) {
+            load_entries(P.shard + lcn * P.nshards, nv, nw);
+            if (deep) {
+                nr0 = n2r0;
+                nrl = n2rl;
+                starts(nr0, nrl, nsa, nsz);
+                if (lcn + P.W < P.nlocal) bracket(lcn + P.W, n2r0, n2rl);
+            } else {
+                bracket(lcn, nr0, nrl);
+            }
+        }
+        int* mark = s_mark[warp];
+#pragma unroll
+        for (int i = lane; i < kChunk; i += 32) mark[i] = -1;
+        __syncwarp();
+        if (deep) {   // the first 64 row starts arrived with the prefetch
+            const int ra = r0 + 1 + lane, rz = r0 + 33 + lane;
+            if (sa >= c0 && sa < c1) atomicMax(&mark[sa - c0], ra);
+            else if (sa < c0) err = true;
+            if (sz >= c0 && sz < c1) atomicMax(&mark[sz - c0], rz);
+            else if (sz < c0) err = true;
+        }
+        for (int rb = r0 + (deep ? 65 : 1); rb <= r_last; rb += 64) {   // (further) row starts
+            const int ra = rb + lane, rz = rb + 32 + lane;
+            const long long ta = ra <= r_last ? __ldg(P.nindex + ra) : LLONG_MAX;
+            const long long tz = rz <= r_last ? __ldg(P.nindex + rz) : LLONG_MAX;
+            if (ta >= c0 && ta < c1) atomicMax(&mark[ta - c0], ra);
+            else if (ta < c0) err = true;
+            if (tz >= c0 && tz < c1) atomicMax(&mark[tz - c0], rz);
+            else if (tz < c0) err = true;
+        }
+        __syncwarp();
+        int row[kItems];
+#pragma unroll
+        for (int k = 0; k < kItems; ++k) row[k] = mark[p0 + k];
+        // inclusive max-scan over the warp's 128 positions
+#pragma unroll
+        for (int k = 1; k < kItems; ++k) row[k] = max(row[k], row[k - 1]);
+        int incl = row[kItems - 1];
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int y = __shfl_up_sync(kFull, incl, o);
+            if (lane >= o) incl = max(incl, y);
+        }
+        int excl = __shfl_up_sync(kFull, incl, 1);
+        if (lane == 0) excl = r0;                 // position 0 belongs to row r0
+#pragma unroll
+        for (int k = 0; k < kItems; ++k) row[k] = max(row[k], max(excl, r0));
+
+        if (PH == 1 && P.zero_mst) {   // every in_mst byte is written once, here (Alg. 1 "not in MST")
+            if (p0 + kItems <= len) {
+                __stcs(reinterpret_cast<unsigned*>(P.in_mst + c0 + p0), 0u);
+            } else {
+#pragma unroll
+                for (int k = 0; k < kItems; ++k)
+                    if (p0 + k < len) P.in_mst[c0 + p0 + k] = 0;
+            }
+        }
+        bool cand[kItems];
+#pragma unroll
+        for (int k = 0; k < kItems; ++k) {
+            const bool valid = p0 + k < len;
+            const bool in_range = (unsigned)vv[k] < (unsigned)P.n;
+            if (valid && !in_range) err = true;
+            const bool canon = valid && in_range && row[k] < vv[k];   // L4: one direction only
+            const bool heavy = filtered && ww[k] >= T;                // L6 threshold condition
+            if (PH == 1) {
+                canon_cnt += canon;
+                heavy_cnt += (canon && heavy);
+                cand[k] = canon && !heavy;
+            } else {
+                cand[k] = canon && heavy;
+            }
+        }
+        int pk[kItems], qk[kItems];
+#pragma unroll
+        for (int k = 0; k < kItems; ++k) {
+            pk[k] = row[k];
+            qk[k] = vv[k];
+        }
+        if (PH == 2) {   // set(v), set(n): one load each after k_flatten
+#pragma unroll
+            for (int k = 0; k < kItems; ++k) {
+                if (cand[k] && giant >= 0 && ((vb >> k) & 1u) &&
+                    ((__ldg(P.giant_bits + (row[k] >> 5)) >> (row[k] & 31)) & 1)) {
+                    pk[k] = qk[k] = giant;                    // both ends in the largest set: filtered
+                } else if (cand[k]) {
+                    pk[k] = (k > 0 && cand[k - 1] && row[k] == row[k - 1]) ? -1 : __ldca(D.par(row[k]));
+                    qk[k] = __ldca(D.par(vv[k]));
+                }
+            }
+#pragma unroll
+            for (int k = 1; k < kItems; ++k)
+                if (pk[k] == -1) pk[k] = pk[k - 1];
+            if (!P.flatten) {
+#pragma unroll
+                for (int k = 0; k < kItems; ++k) {
+                    if (cand[k]) {
+                        pk[k] = find_root(D, pk[k], P.halving != 0);
+                        qk[k] = find_root(D, qk[k], P.halving != 0);
+                    }
+                }
+            }
+        }
+#pragma unroll
+        for (int k = 0; k < kItems; ++k) {
+            const long long j = c0 + p0 + k;
+            t[k] = make_int4(pk[k], qk[k], ww[k], (int)(unsigned)j);
+            keep[k] = cand[k] && pk[k] != qk[k];                  // phase 2: the filter
+        }
+        // L19-21: the lane's entries come in row order, so merge equal p first
+        long long best = kInf;
+        int bp = -1;
+#pragma unroll
+        for (int k = 0; k < kItems; ++k) {
+            if (!keep[k]) continue;
+            const long long key = make_key(t[k].z, (unsigned)t[k].w);   // L19 val <- e_w : e_id
+            if (t[k].x != bp) {
+                if (bp >= 0) record_min(D.k(bp), best, guard);
+                bp = t[k].x;
+                best = key;
+            } else {
+                best = min(best, key);
+            }
+        }
+        if (bp >= 0) record_min(D.k(bp), best, guard);
+#pragma unroll
+        for (int k = 0; k < kItems; ++k)
+            if (keep[k]) record_min(D.k(t[k].y), make_key(t[k].z, (unsigned)t[k].w), guard);
+    }
+    if (PH == 2 && lc + P.W < P.nlocal) nvb = vbits(nv);   // next chunk's far-end bits
+    // L7: append the chunk's tuples to the warp's region
+    unsigned m[kItems];
+    int off[kItems];
+    int tot = 0;
+#pragma unroll
+    for (int i = 0; i < kItems; ++i) {
+        m[i] = __ballot_sync(kFull, keep[i]);
+        off[i] = tot;
+        tot += __popc(m[i]);
+    }
+    const unsigned lt = (1u << lane) - 1u;
+#pragma unroll
+    for (int i = 0; i < kItems; ++i)
+        if (keep[i]) __stcg(out + cnt + off[i] + __popc(m[i] & lt), t[i]);
+    cnt += tot;
+    }
+    if (err) atomicExch(&P.st->status, ECL_MST_ERR_INPUT);
+    if (PH == 1) {   // |E| and the deferred count of this warp's chunks
+        canon_cnt = warp_sum(canon_cnt);
+        heavy_cnt = warp_sum(heavy_cnt);
+    }
+    if (lane == 0) P.region[w] = make_int4(cnt, canon_cnt, heavy_cnt, 0);
+}
+
+}  // namespace eclmst

@@ -1,0 +1,369 @@
+// rounds.cuh -- the round loop: k_flatten / k_giant (before phase 2), the
+// worklist views, pass A (Alg. 2 L14-23), pass B (L27-31 + L34-37), the
+// persistent cooperative k_rounds kernel and k_finalize.
+#pragma once
+
+#include "common.cuh"
+
+namespace eclmst {
+
+// ---------------------------------------------------------------------------
+// k_flatten: parent[v] = find(v) before the phase-2 populate, so the phase-2
+// populate can use parent[x] as set(x) with one load.  Two launches: stage 1
+// compresses with path halving from every vertex (fast, but a halving store
+// of one thread can land after another thread's final root store and leave
+// a vertex one or two hops from its root); stage 2 finishes exactly with
+// owner-only pointer jumping (each slot written by the thread that owns it,
+// reads through L2 to see the others' progress), cheap on the short paths
+// stage 1 leaves.  Roots never change here.
+// ---------------------------------------------------------------------------
+template <int STAGE>
+__global__ void __launch_bounds__(256) k_flatten(Params P) {
+    if (!phase2_needed(P) || !P.flatten) return;
+    const long long stride = (long long)gridDim.x * blockDim.x;
+    const DS D = ds_of(P);
+    const int lane = threadIdx.x & 31;
+    const int giant = (STAGE == 2 && P.giant_bits) ? __ldcg(&P.in->giant) : -1;
+    // warps walk 32 consecutive vertices together (stage 2 ballots the bitmap)
+    for (long long base = (long long)blockIdx.x * blockDim.x + threadIdx.x - lane; base < P.n; base += stride) {
+        const long long v = base + lane;
+        const bool valid = v < P.n;
+        if (STAGE == 1) {
+            // fast, racy compression: path halving by everybody (ends close
+            // to, but not always exactly at, one hop)
+            if (valid) {
+                const int r = find_root(D, (int)v, true);
+                if (r != (int)v) *D.par(v) = r;
+            }
+        } else {
+            // exact: owner-only pointer jumping over the now-short paths
+            int p = valid ? __ldcg(D.par(v)) : -1;
+            while (valid) {
+                const int pp = __ldcg(D.par(p));
+                if (pp == p) break;
+                __stcg(D.par(v), pp);
+                p = pp;
+            }
+            if (P.giant_bits) {
+                const unsigned bits = __ballot_sync(kFull, valid && p == giant);
+                if (lane == 0) P.giant_bits[base >> 5] = bits;
+            }
+        }
+    }
+}
+
+// After phase 1 most vertices of a graph whose light edges percolate (C3-C5)
+// sit in ONE set.  Find its root by a majority vote over sampled vertices;
+// k_flatten<2> then writes a bitmap of its members, and the phase-2 populate
+// filters an edge with both ends in it from the bitmap (n/8 bytes, L2
+// resident) instead of two random parent loads.
+__global__ void __launch_bounds__(256) k_giant(Params P) {
+    __shared__ int s_r[1024];
+    if (!phase2_needed(P) || !P.flatten || !P.giant_bits) return;
+    const DS D = ds_of(P);
+    for (int i = threadIdx.x; i < 1024; i += blockDim.x) {
+        const long long v = (long long)(splitmix64(0x6A09E667F3BCC909ull + (unsigned long long)i) % (unsigned long long)P.n);
+        s_r[i] = find_root(D, (int)v, false);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        int cand = -1, votes = 0;                 // Boyer-Moore majority vote
+        for (int i = 0; i < 1024; ++i) {
+            if (votes == 0) { cand = s_r[i]; votes = 1; }
+            else votes += (s_r[i] == cand) ? 1 : -1;
+        }
+        int cnt = 0;
+        for (int i = 0; i < 1024; ++i) cnt += s_r[i] == cand;
+        P.in->giant = cnt >= 256 ? cand : -1;     // worth a bitmap only if it holds >= 1/4
+    }
+}
+
+// ---------------------------------------------------------------------------
+// rounds: pass A / pass B over the CTA's arena
+// ---------------------------------------------------------------------------
+
+// A CTA's worklist as a sequence of 128-tuple chunks.  Right after populate
+// it is the CTA's share of the populate regions (regions b, b+G, ..., each a
+// dense run of region[w].x tuples; chunk j maps to a region by a binary
+// search over the shared prefix s_pre) -- RegionSrc; after a pass A it is one
+// compact run of cnt tuples -- CompactSrc.  Two types, so each pass is
+// compiled once per mode and carries only the registers that mode needs.
+struct CompactSrc {
+    const int4* base;
+    int cnt;
+    int nloc;
+    __device__ __forceinline__ const int4* get(const Params&, int j, int& count) const {
+        count = min(kChunk, cnt - j * kChunk);
+        return base + (long long)j * kChunk;
+    }
+};
+
+struct RegionSrc {
+    const int* s_pre;   // shared memory: chunk prefix per region (nreg + 1)
+    const int* s_rcnt;  // shared memory: tuples per region
+    int nreg;
+    int nloc;
+    int first_w;
+    __device__ __forceinline__ const int4* get(const Params& P, int j, int& count) const {
+        int lo = 0, hi = nreg;
+        while (hi - lo > 1) {
+            const int mid = (lo + hi) >> 1;
+            if (s_pre[mid] <= j) lo = mid;
+            else hi = mid;
+        }
+        const int off = j - s_pre[lo];
+        count = min(kChunk, s_rcnt[lo] - off * kChunk);
+        return P.wl0 + (long long)(first_w + lo * P.G) * P.rcap + (long long)off * kChunk;
+    }
+};
+
+__device__ __forceinline__ CompactSrc compact_src(const int4* base, int cnt) {
+    CompactSrc S;
+    S.base = base;
+    S.cnt = cnt;
+    S.nloc = (cnt + kChunk - 1) / kChunk;
+    return S;
+}
+
+// the populate output of CTA b: regions w = b, b + G, ...  Loads the region
+// counts into shared memory, builds the chunk prefix, and adds the kept,
+// canonical and deferred counts to the stats (phase 1 counters only if
+// count_phase1).  Every thread of the CTA must call it.
+__device__ __forceinline__ RegionSrc region_src(const Params& P, int b, int* s_pre, int* s_rcnt,
+                                                long long (*s_red)[kWarps], int64_t* live_slot,
+                                                bool count_phase1) {
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    RegionSrc R;
+    R.s_pre = s_pre;
+    R.s_rcnt = s_rcnt;
+    R.nreg = b < P.W ? (P.W - b + P.G - 1) / P.G : 0;
+    R.first_w = b;
+    long long canon = 0, heavy = 0;
+    for (int k = tid; k < R.nreg; k += kBlock) {
+        const int4 r = P.region[b + k * P.G];
+        s_rcnt[k] = r.x;
+        canon += r.y;
+        heavy += r.z;
+    }
+    canon = warp_sum(canon);
+    heavy = warp_sum(heavy);
+    if (lane == 0) {
+        s_red[1][warp] = canon;
+        s_red[2][warp] = heavy;
+    }
+    __syncthreads();
+    if (tid == 0) {
+        long long kept = 0;
+        int pre = 0;
+        for (int k = 0; k < R.nreg; ++k) {
+            s_pre[k] = pre;
+            pre += (s_rcnt[k] + kChunk - 1) / kChunk;
+            kept += s_rcnt[k];
+        }
+        s_pre[R.nreg] = pre;
+        canon = heavy = 0;
+        for (int w2 = 0; w2 < kWarps; ++w2) {
+            canon += s_red[1][w2];
+            heavy += s_red[2][w2];
+        }
+        if (kept) atomicAdd(reinterpret_cast<unsigned long long*>(live_slot), (unsigned long long)kept);
+        if (count_phase1) {
+            if (canon) atomicAdd(reinterpret_cast<unsigned long long*>(&P.st->canonical_edges), (unsigned long long)canon);
+            if (heavy) atomicAdd(reinterpret_cast<unsigned long long*>(&P.st->heavy_edges), (unsigned long long)heavy);
+        }
+    }
+    __syncthreads();
+    R.nloc = s_pre[R.nreg];
+    return R;
+}
+
+// L14-23 of one round over the CTA's worklist: S -> out (compact).
+template <class SRC>
+__device__ __forceinline__ void passA(const Params& P, const SRC& S, int4* __restrict__ out, int* s_out,
+                                      bool guard) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const bool halving = P.halving != 0;
+    const DS D = ds_of(P);
+    for (int k = warp; k < S.nloc; k += kWarps) {
+        int count;
+        const int4* __restrict__ in = S.get(P, k, count);
+        int4 t[kItems];
+        bool keep[kItems];
+#pragma unroll
+        for (int i = 0; i < kItems; ++i) {
+            const int idx = i * 32 + lane;
+            keep[i] = idx < count;
+            t[i] = keep[i] ? __ldcs(in + idx) : make_int4(0, 0, 0, 0);
+        }
+        int px[kItems], qx[kItems];
+#pragma unroll
+        for (int i = 0; i < kItems; ++i) {
+            if (keep[i]) {
+                px[i] = __ldca(D.par(t[i].x));
+                qx[i] = __ldca(D.par(t[i].y));
+            }
+        }
+#pragma unroll
+        for (int i = 0; i < kItems; ++i) {
+            if (keep[i]) {
+                const int p = find_from(D, t[i].x, px[i], halving);        // L15
+                const int q = find_from(D, t[i].y, qx[i], halving);        // L16
+                keep[i] = p != q;                                          // L17
+                t[i].x = p;                                                // L18: implicit
+                t[i].y = q;                                                //      path compression
+            }
+        }
+#pragma unroll
+        for (int i = 0; i < kItems; ++i) {
+            if (keep[i]) {
+                const long long key = make_key(t[i].z, (unsigned)t[i].w); // L19
+                record_min(D.k(t[i].x), key, guard);                      // L20
+                record_min(D.k(t[i].y), key, guard);                      // L21
+            }
+        }
+        warp_emit(t, keep, out, s_out);                                   // L18
+    }
+}
+
+// L27-31 (+ L34-37): check, join, mark over the CTA's worklist.
+template <class SRC>
+__device__ __forceinline__ void passB(const Params& P, const SRC& S, long long& wsum, long long& wcnt) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    const DS D = ds_of(P);
+    for (int k = warp; k < S.nloc; k += kWarps) {
+        int count;
+        const int4* __restrict__ in = S.get(P, k, count);
+        int4 t[kItems];
+        bool ok[kItems];
+#pragma unroll
+        for (int i = 0; i < kItems; ++i) {
+            const int idx = i * 32 + lane;
+            ok[i] = idx < count;
+            t[i] = ok[i] ? __ldcg(in + idx) : make_int4(0, 0, 0, 0);
+        }
+        // Only the id half of each slot is compared: ids are unique per
+        // edge, so id equality is key equality (and inf's id half, 2^32-1,
+        // is never a valid id).  L1 is fine: K[p] only changes when p's own
+        // winner resets it.
+        unsigned kp[kItems], kq[kItems];
+#pragma unroll
+        for (int i = 0; i < kItems; ++i) {
+            if (ok[i]) {
+                kp[i] = __ldca(reinterpret_cast<const unsigned*>(D.k(t[i].x)));
+                kq[i] = __ldca(reinterpret_cast<const unsigned*>(D.k(t[i].y)));
+            }
+        }
+#pragma unroll
+        for (int i = 0; i < kItems; ++i) {
+            if (!ok[i]) continue;
+            const bool wp = kp[i] == (unsigned)t[i].w, wq = kq[i] == (unsigned)t[i].w;   // L29
+            if (wp || wq) {
+                const int p = t[i].x, q = t[i].y;
+                // L30 join: each set hooks along its own lightest edge;
+                // a mutual pair keeps the smaller representative as root.
+                if (wp && !(wq && p < q)) __stcg(D.par(p), q);
+                if (wq && !(wp && q < p)) __stcg(D.par(q), p);
+                if (wp) __stcg(D.k(p), kInf);                          // L35
+                if (wq) __stcg(D.k(q), kInf);                          // L36
+                P.in_mst[(unsigned)t[i].w] = 1;                        // L31
+                wsum += t[i].z;
+                wcnt += 1;
+            }
+        }
+    }
+}
+
+// guard policy for pass A.  "auto" guards when edges crowd onto few
+// sets -- each set with a live edge produced exactly one winner last round
+// (mutual pairs: one for two sets), so live / winners estimates the number of
+// edges per set that would atomicMin the same slot -- or when the key array
+// is far larger than L2 (n >= 2^25: every unguarded atomic on a random slot
+// is a DRAM read-modify-write, a guard miss only a read).  Measured: C5 and
+// C4 gain, C2/C3 lose with guards in every round.
+__device__ __forceinline__ bool use_guard(const Params& P, long long live, long long winners) {
+    if (P.guards >= 0) return P.guards != 0;
+    return live > 8 * winners || P.n >= (1 << 25);
+}
+
+template <int PH>
+__global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
+    cg::grid_group grid = cg::this_grid();
+    __shared__ int s_out;
+    __shared__ long long s_red[3][kWarps];
+    __shared__ int s_pre[kMaxRegionsPerCta + 1];
+    __shared__ int s_rcnt[kMaxRegionsPerCta];
+    const int tid = threadIdx.x, lane = tid & 31;
+    const bool b0 = blockIdx.x == 0;
+    ecl_mst_stats* st = P.st;
+    if (PH == 2 && !phase2_needed(P)) return;
+    int g = (PH == 1) ? 0 : __ldcg(&P.in->g_end) + 1;
+    if (g >= ECL_MST_MAX_ROUNDS) {
+        if (b0 && tid == 0) atomicExch(&st->status, ECL_MST_ERR_INPUT);
+        return;
+    }
+    stamp(P, 4 + 2 * g);                      // populate done
+    const int b = blockIdx.x;
+    int4* wl[2] = {P.wl0 + (long long)b * P.cap, P.wl1 + (long long)b * P.cap};
+    // the populate output of this CTA: regions w = b, b + G, ... (region mode)
+    const RegionSrc R = region_src(P, b, s_pre, s_rcnt, s_red, &st->live[g], PH == 1);
+    if (b0 && tid == 0 && PH == 2) st->phase2_round = g;
+    trace_cta(P, 4 + 2 * g);
+    grid.sync();
+    long long wsum = 0, wcnt = 0;
+    int cur = 0;
+    bool overflow = false;
+    long long L = __ldcg(&st->live[g]);
+    CompactSrc C = compact_src(wl[0], 0);
+    // one round: pass B over S, then pass A from S into the other worklist
+    auto round = [&](const auto& S) {
+        const long long w0 = wcnt;
+        passB(P, S, wsum, wcnt);
+        const long long d = warp_sum(wcnt - w0);
+        if (lane == 0 && d) atomicAdd(reinterpret_cast<unsigned long long*>(&st->winners[g]), (unsigned long long)d);
+        if (tid == 0) s_out = 0;
+        trace_cta(P, 5 + 2 * g);
+        grid.sync();
+        stamp(P, 5 + 2 * g);
+        if (g + 1 >= ECL_MST_MAX_ROUNDS) {
+            overflow = true;
+            return false;
+        }
+        const bool guard = use_guard(P, L, __ldcg(&st->winners[g]));
+        ++g;
+        passA(P, S, wl[cur ^ 1], &s_out, guard);
+        cur ^= 1;
+        __syncthreads();
+        C = compact_src(wl[cur], s_out);
+        if (tid == 0 && C.cnt) atomicAdd(reinterpret_cast<unsigned long long*>(&st->live[g]), (unsigned long long)C.cnt);
+        trace_cta(P, 4 + 2 * g);
+        grid.sync();
+        stamp(P, 4 + 2 * g);
+        L = __ldcg(&st->live[g]);
+        return true;
+    };
+    if (L > 0 && round(R))
+        while (L > 0 && round(C)) {
+        }
+    const long long s = warp_sum(wsum), c = warp_sum(wcnt);
+    if (lane == 0) {
+        if (s) atomicAdd(reinterpret_cast<unsigned long long*>(&st->total_weight), (unsigned long long)s);
+        if (c) atomicAdd(reinterpret_cast<unsigned long long*>(&st->msf_edges), (unsigned long long)c);
+    }
+    if (b0 && tid == 0) {
+        P.in->g_end = g;
+        st->rounds = g + 1;
+        if (overflow) atomicExch(&st->status, ECL_MST_ERR_INPUT);
+    }
+}
+
+__global__ void k_finalize(Params P) {
+    if (threadIdx.x == 0) {
+        ecl_mst_stats* st = P.st;
+        st->t_ns[2] = (long long)globaltimer_ns();
+        const int status = *reinterpret_cast<volatile int*>(&st->status);
+        *P.total_out = status ? LLONG_MIN : *reinterpret_cast<volatile long long*>(&st->total_weight);
+    }
+}
+
+
+}  // namespace eclmst
