@@ -72,7 +72,10 @@ typedef struct ecl_mst_options {
     uint64_t seed;           /* seed of the threshold sample */
     int32_t threshold_samples; /* sample size S for threshold_mode 0 (paper: 20; default
                                   1024 -- same target, far less variance; <= 4096) */
-    int32_t reserved;
+    int32_t populate_order;  /* which CSR chunks each populate warp takes (a performance knob; the
+                                result does not depend on it): 1 interleaved (chunks w, w + W, ...),
+                                2 one contiguous slice per warp, 3 contiguous in phase 1 and
+                                interleaved in phase 2; 0 auto (currently 3) */
 } ecl_mst_options;
 
 /* per-run statistics written by the device into the workspace */

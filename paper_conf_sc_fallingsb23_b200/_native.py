@@ -36,7 +36,7 @@ class EclMstOptions(ctypes.Structure):
         ("trace", ctypes.c_int32),
         ("seed", ctypes.c_uint64),
         ("threshold_samples", ctypes.c_int32),
-        ("reserved", ctypes.c_int32),
+        ("populate_order", ctypes.c_int32),
     ]
 
 

@@ -77,6 +77,7 @@ struct Params {
     long long cap;                    // tuples per arena (k_rounds worklists)
     int W;                            // populate warps = regions of wl0
     long long rcap;                   // tuples per region
+    int pop_contig;                   // bit PH-1: populate<PH> walks contiguous slices of rcap/kChunk chunks
     const long long* __restrict__ nindex;
     const int* __restrict__ nlist;
     const int* __restrict__ eweight;

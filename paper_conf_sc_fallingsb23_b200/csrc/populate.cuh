@@ -106,7 +106,7 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
     // the density of u < v entries drifts along the rows) and appends its
     // tuples densely to its own region: no atomics, no CTA barrier.
     const int w = blockIdx.x * kPopWarps + warp;
-    if (w >= P.W) return;
+    if (w >= P.W) return;   // (sharded path: partial last CTA)
     int4* const out = P.wl0 + (long long)w * P.rcap;
     int cnt = 0, canon_cnt = 0, heavy_cnt = 0;
     bool err = false;
@@ -162,16 +162,24 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
     int nr0 = 0, nrl = 0, n2r0 = 0, n2rl = 0, nv[kItems], nw[kItems];
     long long nsa = LLONG_MAX, nsz = LLONG_MAX;
     unsigned nvb = 0;
-    if (w < P.nlocal) {
-        bracket(w, nr0, nrl);
-        load_entries(P.shard + (long long)w * P.nshards, nv, nw);
+    // the warp's chunks: interleaved w, w + W, ... or the contiguous slice
+    // [w B, (w + 1) B) with B = rcap / kChunk (see P.pop_contig)
+    const bool contig = (P.pop_contig >> (PH - 1)) & 1;
+    const long long span = P.rcap / kChunk;
+    const long long step = contig ? 1 : P.W;
+    const long long lc0 = contig ? (long long)w * span : w;
+    const long long lend = contig ? min(lc0 + span, P.nlocal) : P.nlocal;
+    auto nxt = [&](long long lc) { return lc + step; };
+    if (lc0 < lend) {
+        bracket(lc0, nr0, nrl);
+        load_entries(P.shard + lc0 * P.nshards, nv, nw);
         if (deep) {
             starts(nr0, nrl, nsa, nsz);
-            if (w + P.W < P.nlocal) bracket(w + P.W, n2r0, n2rl);
+            if (nxt(lc0) < lend) bracket(nxt(lc0), n2r0, n2rl);
         }
         nvb = vbits(nv);
     }
-    for (long long lc = w; lc < P.nlocal; lc += P.W) {
+    for (long long lc = lc0; lc < lend; lc = nxt(lc)) {
     const long long c = P.shard + lc * P.nshards;
     bool keep[kItems];
     int4 t[kItems];
@@ -191,14 +199,14 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
             vv[k] = nv[k];
             ww[k] = nw[k];
         }
-        const long long lcn = lc + P.W;
-        if (lcn < P.nlocal) {
+        const long long lcn = nxt(lc);
+        if (lcn < lend) {
             load_entries(P.shard + lcn * P.nshards, nv, nw);
             if (deep) {
                 nr0 = n2r0;
                 nrl = n2rl;
                 starts(nr0, nrl, nsa, nsz);
-                if (lcn + P.W < P.nlocal) bracket(lcn + P.W, n2r0, n2rl);
+                if (nxt(lcn) < lend) bracket(nxt(lcn), n2r0, n2rl);
             } else {
                 bracket(lcn, nr0, nrl);
             }
@@ -322,7 +330,7 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
         for (int k = 0; k < kItems; ++k)
             if (keep[k]) record_min(D.k(t[k].y), make_key(t[k].z, (unsigned)t[k].w), guard);
     }
-    if (PH == 2 && lc + P.W < P.nlocal) nvb = vbits(nv);   // next chunk's far-end bits
+    if (PH == 2 && nxt(lc) < lend) nvb = vbits(nv);   // next chunk's far-end bits
     // L7: append the chunk's tuples to the warp's region
     unsigned m[kItems];
     int off[kItems];

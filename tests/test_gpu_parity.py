@@ -94,6 +94,8 @@ def test_config_small(eclmst, name):
     dict(seed=1), dict(seed=12345), dict(path_halving=0), dict(max_ctas=1), dict(max_ctas=7),
     dict(atomic_guards=0), dict(atomic_guards=1), dict(flatten=0), dict(flatten=0, path_halving=0), dict(trace=1),
     dict(threshold_samples=20), dict(threshold_samples=4096, seed=7),
+    dict(populate_order=1), dict(populate_order=2), dict(populate_order=3), dict(populate_order=2, max_ctas=3),
+    dict(populate_order=1, max_ctas=2),
 ])
 @pytest.mark.parametrize("name", ["rmat", "uniform", "road"])
 def test_knobs_give_identical_msf(eclmst, name, opts):
