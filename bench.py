@@ -29,7 +29,6 @@ sys.path.insert(0, ROOT)
 import torch  # noqa: E402
 
 PEAKS_FILE = os.path.join(ROOT, "MEASURED_PEAKS.json")
-PROFILE_SUMMARY = os.path.join(ROOT, "profiles", "ncu_summary_latest.json")
 # k_init, k_populate<1>, k_rounds<1>, k_finalize; with filtering also k_flatten<1>, k_flatten<2>,
 # k_populate<2>, k_rounds<2>
 LAUNCHES_UNFILTERED, LAUNCHES_FILTERED = 4, 8
@@ -211,13 +210,18 @@ def load_peaks():
         return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
-def load_traffic():
-    try:
-        with open(PROFILE_SUMMARY) as f:
-            s = json.load(f)
-        return s
-    except (OSError, ValueError):
-        return None
+def load_traffic(workload):
+    """The committed ncu --set full summary of this workload (profiles/ncu_summary_*.json), or None."""
+    import glob
+    for path in sorted(glob.glob(os.path.join(ROOT, "profiles", "ncu_summary_*.json"))):
+        try:
+            with open(path) as f:
+                s = json.load(f)
+        except (OSError, ValueError):
+            continue
+        if s.get("workload") == workload:
+            return s
+    return None
 
 
 # ---------------------------------------------------------------------------
@@ -344,6 +348,7 @@ def main():
 
     # ---- e2e through the host C-ABI call (pinned host buffers, copies timed) ----
     e2e = None
+    in_mst_h = None
     if not args.no_e2e and use_dist:
         # sharded e2e through the public API: pinned host CSR -> device, run, mask -> host
         h_idx = g.nindex.cpu().pin_memory()
@@ -376,6 +381,10 @@ def main():
                "ms_per_step": e_ms, "same_result": tot_h == result_total,
                "path": "ecl_mst_dist_device with pinned host->device copies (every rank holds the CSR)"}
     if not args.no_e2e and not use_dist:
+        # the host path allocates its own device copies and workspace: free ours first (C5: 65 GB)
+        in_mst_h = in_mst.cpu()
+        del ws, flush
+        torch.cuda.empty_cache()
         h_idx = g.nindex.cpu().pin_memory()
         h_list = g.nlist.cpu().pin_memory()
         h_w = g.eweight.cpu().pin_memory()
@@ -411,7 +420,7 @@ def main():
             omask, ototal, _ = oracle.kruskal(hn, hidx, hlist, hw)
             o_s = time.perf_counter() - t0
             if not args.no_parity:
-                parity = bool(ototal == result_total and np.array_equal(omask, in_mst.cpu().numpy()))
+                parity = bool(ototal == result_total and np.array_equal(omask, (in_mst_h if in_mst_h is not None else in_mst.cpu()).numpy()))
             sample_desc = f"whole {g.name} graph, one serial C Kruskal run (oracle/kruskal.c)"
             sample_M = M
         else:
@@ -439,9 +448,9 @@ def main():
         ab["total_step"] = ab["total"]
         dominant = "total_step"
     achieved = ab[dominant] / (kern_ms.get(dominant, ms_max) / 1e3) / 1e9
-    prof = load_traffic()
+    prof = load_traffic(g.name)
     traffic = None
-    if prof and prof.get("workload") == g.name:
+    if prof:
         traffic = prof.get("dram_bytes_per_launch", {}).get(dominant)
     value = M / (ms_max / 1e3)   # one graph per step, whatever N (strong scaling)
     line = {

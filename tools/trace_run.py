@@ -24,9 +24,11 @@ def main():
     ap.add_argument("--size", default="full")
     ap.add_argument("--opt", action="append", default=[])
     ap.add_argument("--runs", type=int, default=3)
+    ap.add_argument("--ov", action="append", default=[], help="generator override k=v (e.g. width=3000)")
     args = ap.parse_args()
     dev = torch.device("cuda:0")
-    g = synth.make_config(args.config, args.size, device=dev)
+    ov = {k: (float(v) if "." in v else int(v)) for k, v in (o.split("=") for o in args.ov)}
+    g = synth.make_config(args.config, args.size, device=dev, **ov)
     kw = {k: int(v) for k, v in (o.split("=") for o in args.opt)}
     kw["trace"] = 1
     opts = eclmst.default_options(**kw)
