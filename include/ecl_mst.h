@@ -44,7 +44,7 @@
 extern "C" {
 #endif
 
-#define ECL_MST_ABI_VERSION 1
+#define ECL_MST_ABI_VERSION 2
 
 /* status codes */
 #define ECL_MST_OK 0
@@ -54,7 +54,7 @@ extern "C" {
 #define ECL_MST_ERR_WORKSPACE (-4) /* workspace too small or misaligned */
 #define ECL_MST_ERR_INPUT (-5)     /* the device found an inconsistent CSR (stats.status) */
 
-#define ECL_MST_MAX_ROUNDS 128     /* global round slots (<= ceil(log2 n)+1 per phase) */
+#define ECL_MST_MAX_ROUNDS 128     /* global round slots (<= ceil(log2 n)+1 per phase and sub-phase) */
 
 /* knobs; every setting returns the identical MSF (tests check this) */
 typedef struct ecl_mst_options {
@@ -76,6 +76,17 @@ typedef struct ecl_mst_options {
                                 result does not depend on it): 1 interleaved (chunks w, w + W, ...),
                                 2 one contiguous slice per warp, 3 contiguous in phase 1 and
                                 interleaved in phase 2; 0 auto (currently 3) */
+    int32_t refilter;        /* crowded rounds (live edges >> sets, e.g. RMAT/uniform after the
+                                giant set forms): re-apply the paper's threshold filter (P:143,
+                                P:152) to the live worklist -- edges below a sampled threshold T'
+                                run to completion first, the rest are deferred and filtered by
+                                set(u) != set(v) afterwards.  -1 (default) auto: when >= 2^20 live
+                                tuples and > 16 per MSF edge of the last round; 0 never; 1 whenever
+                                live > 4 x last round's MSF edges (tests).  Same MSF either way. */
+    int32_t filter_c;        /* c of P:143: the threshold targets the c|V| lightest CSR entries.
+                                0 (default) = 4, "we use c = 4 in our code"; P:394 aims
+                                for 3; "values between 2 and 4 seem to work well".  Only
+                                speed depends on it. */
 } ecl_mst_options;
 
 /* per-run statistics written by the device into the workspace */
@@ -87,7 +98,7 @@ typedef struct ecl_mst_stats {
     int32_t phase2_round;    /* first global round of phase 2 (-1 if none) */
     int32_t grid;            /* CTAs of the persistent launch */
     int32_t block;           /* threads per CTA */
-    int32_t reserved;
+    int32_t refilters;       /* crowded-round splits taken (opts.refilter); each adds one sub-phase */
     int64_t total_weight;
     int64_t msf_edges;
     int64_t canonical_edges; /* |E| = #{j : u < nlist[j]} */

@@ -15,6 +15,7 @@ import torch
 from . import build as _build
 
 MAX_ROUNDS = 128
+ABI_VERSION = 2          # include/ecl_mst.h ECL_MST_ABI_VERSION
 
 OK = 0
 ERR_INVALID = -1
@@ -37,6 +38,8 @@ class EclMstOptions(ctypes.Structure):
         ("seed", ctypes.c_uint64),
         ("threshold_samples", ctypes.c_int32),
         ("populate_order", ctypes.c_int32),
+        ("refilter", ctypes.c_int32),
+        ("filter_c", ctypes.c_int32),
     ]
 
 
@@ -49,7 +52,7 @@ class EclMstStats(ctypes.Structure):
         ("phase2_round", ctypes.c_int32),
         ("grid", ctypes.c_int32),
         ("block", ctypes.c_int32),
-        ("reserved", ctypes.c_int32),
+        ("refilters", ctypes.c_int32),
         ("total_weight", ctypes.c_int64),
         ("msf_edges", ctypes.c_int64),
         ("canonical_edges", ctypes.c_int64),
@@ -116,7 +119,7 @@ def load(build_if_missing: bool = False):
     L.ecl_mst_dist_device.restype = ctypes.c_int
     L.ecl_mst_dist_device.argtypes = [vp, i32, i32, i64, vp, vp, vp, vp, vp, vp, sz,
                                       ctypes.POINTER(EclMstOptions), vp]
-    if L.ecl_mst_abi_version() != 1:
+    if L.ecl_mst_abi_version() != ABI_VERSION:
         raise ImportError("libeclmst.so ABI version mismatch")
     _lib = L
     return L
@@ -217,6 +220,7 @@ def ecl_mst_read_stats(workspace, stream=None) -> dict:
     return {
         "status": st.status, "filtered": bool(st.filtered), "threshold": st.threshold,
         "rounds": st.rounds, "phase2_round": st.phase2_round, "grid": st.grid, "block": st.block,
+        "refilters": st.refilters,
         "total_weight": st.total_weight, "msf_edges": st.msf_edges,
         "canonical_edges": st.canonical_edges, "heavy_edges": st.heavy_edges,
         "live": list(st.live[:R]), "winners": list(st.winners[:R]),

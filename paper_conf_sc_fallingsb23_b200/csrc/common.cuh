@@ -22,6 +22,8 @@ constexpr int kMaxPopWarps = 65536;            // populate warps (= worklist reg
 constexpr int kMaxRegionsPerCta = 256;         // regions a k_rounds CTA starts from
 constexpr int kTraceSlots = 2 * ECL_MST_MAX_ROUNDS + 4;
 constexpr int kMaxSamples = 4096;              // threshold sample size cap
+constexpr int kSplitSamples = 512;             // crowded-round threshold: about this many samples
+constexpr int kSplitSampleSlots = 1024;        // sample slots (max(1, 512 / G) per CTA, first CTAs)
 static_assert(kMaxGrid == ECL_MST_TRACE_CTAS, "trace layout");
 
 struct Internal {
@@ -30,11 +32,11 @@ struct Internal {
     int g_cur;                         // first global round of the running phase
     int g_end;                         // last global round of the finished phase
     int giant;                         // root of the largest set after phase 1 (-1: none)
-    int pad0;
+    int splits;                        // crowded-round splits taken so far (all phases)
 };
 
 struct Layout {
-    size_t stats, internal, trace, rowstart, region, giant, key, parent, wl0, wl1, total;
+    size_t stats, internal, trace, rowstart, region, giant, samp, key, parent, wl0, wl1, total;
     long long wl_cap;                  // tuples per worklist buffer
 };
 
@@ -61,6 +63,7 @@ static inline Layout layout_for(int64_t n, int64_t M) {
     L.rowstart = off; off = align_up(off + sizeof(int) * (size_t)(nchunks + 1), 256);
     L.region = off;   off = align_up(off + sizeof(int4) * (size_t)kMaxPopWarps, 256);
     L.giant = off;    off = align_up(off + sizeof(unsigned) * (size_t)((n + 31) / 32 + 1), 256);
+    L.samp = off;     off = align_up(off + sizeof(int) * (size_t)kSplitSampleSlots, 256);
     L.key = off;      off = align_up(off + sizeof(long long) * (size_t)n, 256);
     L.parent = off;   off = align_up(off + sizeof(int) * (size_t)n, 256);
     L.wl0 = off;      off = align_up(off + sizeof(int4) * (size_t)L.wl_cap, 256);
@@ -98,9 +101,12 @@ struct Params {
     int threshold_mode;
     int threshold_value;
     int samples;
+    int filter_c;                     // c of P:143 (threshold targets c|V| lightest CSR entries)
     int halving;
     int guards;                       // -1 auto, 0 off, 1 on
     int flatten;
+    int refilter;                     // -1 auto, 0 off, 1 forced (opts.refilter)
+    int* samp;                        // crowded-round weight samples (kSplitSampleSlots)
     // edge sharding (distributed path; single GPU: shard 0 of 1)
     int shard;                        // global shard id
     int nshards;                      // total shards

@@ -109,6 +109,31 @@ __device__ __forceinline__ int warp_emit(const int4 (&t)[kItems], const bool (&k
     return tot;
 }
 
+// Same, for the tuples a crowded-round split defers: they fill the arena from
+// its end downwards ([end - total, end) after the pass, contiguous).
+__device__ __forceinline__ void warp_emit_back(const int4 (&t)[kItems], const bool (&keep)[kItems],
+                                               int4* __restrict__ end, int* s_cnt) {
+    const int lane = threadIdx.x & 31;
+    unsigned m[kItems];
+    int off[kItems];
+    int tot = 0;
+#pragma unroll
+    for (int i = 0; i < kItems; ++i) {
+        m[i] = __ballot_sync(kFull, keep[i]);
+        off[i] = tot;
+        tot += __popc(m[i]);
+    }
+    if (!tot) return;
+    int base = 0;
+    if (lane == 0) base = atomicAdd(s_cnt, tot);
+    base = __shfl_sync(kFull, base, 0);
+    int4* dst = end - base - tot;
+    const unsigned lt = (1u << lane) - 1u;
+#pragma unroll
+    for (int i = 0; i < kItems; ++i)
+        if (keep[i]) __stcg(dst + off[i] + __popc(m[i] & lt), t[i]);
+}
+
 // warp-cooperative 32-ary search: largest r in [0, n) with nindex[r] <= x.
 // Requires nindex[0] <= x; about log32(n) dependent 8-byte loads.
 __device__ __forceinline__ int warp_row_of(const long long* __restrict__ nindex, int n, long long x) {

@@ -129,6 +129,8 @@ void ecl_mst_default_options(ecl_mst_options* o) {
     o->seed = 0x5eedull;
     o->threshold_samples = 1024;
     o->populate_order = 0;
+    o->refilter = -1;
+    o->filter_c = 0;
 }
 
 size_t ecl_mst_workspace_bytes(int64_t n, int64_t M) {
@@ -229,9 +231,12 @@ int ecl_mst_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t* n
     P.threshold_mode = o.threshold_mode;
     P.threshold_value = o.threshold;
     P.samples = o.threshold_samples > 0 ? std::min(o.threshold_samples, kMaxSamples) : 20;
+    P.filter_c = o.filter_c > 0 ? o.filter_c : 4;
     P.halving = o.path_halving ? 1 : 0;
     P.guards = o.atomic_guards < 0 ? -1 : (o.atomic_guards ? 1 : 0);
     P.flatten = o.flatten ? 1 : 0;
+    P.refilter = o.refilter < 0 ? -1 : (o.refilter ? 1 : 0);
+    P.samp = reinterpret_cast<int*>(ws + L.samp);
     P.shard = 0;
     P.nshards = 1;
     P.nlocal = nchunks;
@@ -679,9 +684,12 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
         P.threshold_mode = o.threshold_mode;
         P.threshold_value = o.threshold;
         P.samples = o.threshold_samples > 0 ? std::min(o.threshold_samples, kMaxSamples) : 20;
+        P.filter_c = o.filter_c > 0 ? o.filter_c : 4;
         P.halving = o.path_halving ? 1 : 0;
         P.guards = o.atomic_guards == 0 ? 0 : 1;
         P.flatten = o.flatten ? 1 : 0;
+        P.refilter = 0;                 // the sharded rounds are host-driven (no split)
+        P.samp = nullptr;
         P.shard = shard;
         P.nshards = (int)Pt;
         P.nlocal = nlocal;

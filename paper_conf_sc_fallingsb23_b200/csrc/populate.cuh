@@ -7,6 +7,7 @@
 
 namespace eclmst {
 
+
 // ---------------------------------------------------------------------------
 // k_init: Alg. 1 + chunk start rows + threshold
 // ---------------------------------------------------------------------------
@@ -43,7 +44,7 @@ __global__ void __launch_bounds__(256) k_init(Params P) {
                 s_w[i] = P.eweight[(long long)(h % (unsigned long long)P.M)];
             }
             __syncthreads();
-            long long kpos = ((long long)S * 4LL * P.n) / P.M;
+            long long kpos = ((long long)S * P.filter_c * P.n) / P.M;   // c|V| lightest
             if (kpos > S - 1) kpos = S - 1;
             for (int i = tid; i < S; i += blockDim.x) {
                 const int wi = s_w[i];
@@ -68,6 +69,7 @@ __global__ void __launch_bounds__(256) k_init(Params P) {
             P.in->g_end = 0;
             P.in->done = 0;
             P.in->giant = -1;
+            P.in->splits = 0;
         }
     }
     if (err) atomicExch(&P.st->status, ECL_MST_ERR_INPUT);

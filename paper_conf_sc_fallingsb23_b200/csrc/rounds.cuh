@@ -3,6 +3,8 @@
 // persistent cooperative k_rounds kernel and k_finalize.
 #pragma once
 
+#include <type_traits>
+
 #include "common.cuh"
 
 namespace eclmst {
@@ -177,10 +179,14 @@ __device__ __forceinline__ RegionSrc region_src(const Params& P, int b, int* s_p
     return R;
 }
 
-// L14-23 of one round over the CTA's worklist: S -> out (compact).
-template <class SRC>
+// L14-23 of one round over the CTA's worklist: S -> out (compact).  With a
+// split threshold T < INT_MAX (a crowded round, see split_threshold) only the
+// tuples with w < T record their key and go to the front of `out`; the others
+// are deferred to the back of the arena (ending at out_end, count in *s_def).
+template <bool SPLIT = false, class SRC>
 __device__ __forceinline__ void passA(const Params& P, const SRC& S, int4* __restrict__ out, int* s_out,
-                                      bool guard) {
+                                      bool guard, int T = INT_MAX, int4* out_end = nullptr,
+                                      int* s_def = nullptr) {
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const bool halving = P.halving != 0;
     const DS D = ds_of(P);
@@ -212,6 +218,15 @@ __device__ __forceinline__ void passA(const Params& P, const SRC& S, int4* __res
                 t[i].x = p;                                                // L18: implicit
                 t[i].y = q;                                                //      path compression
             }
+        }
+        if (SPLIT) {   // crowded round: defer w >= T (they record no key)
+            bool heavy[kItems];
+#pragma unroll
+            for (int i = 0; i < kItems; ++i) {
+                heavy[i] = keep[i] && t[i].z >= T;
+                keep[i] = keep[i] && t[i].z < T;
+            }
+            warp_emit_back(t, heavy, out_end, s_def);
         }
 #pragma unroll
         for (int i = 0; i < kItems; ++i) {
@@ -285,13 +300,82 @@ __device__ __forceinline__ bool use_guard(const Params& P, long long live, long 
     return live > 8 * winners || P.n >= (1 << 25);
 }
 
+// ---------------------------------------------------------------------------
+// crowded rounds.  Once a giant set forms (RMAT, uniform graphs), most live
+// edges join a handful of huge sets: C5 keeps ~78 M live tuples for six
+// rounds that add 77 K, 11 K, ..., 3 MSF edges.  Every such round rereads all
+// of them to find one minimum per set.  The paper's own remedy for the whole
+// graph -- process the edges below a sampled threshold first, then filter the
+// rest by set(u) != set(v) -- applies to the live worklist as
+// well: the light part runs to completion, then the deferred part is
+// filtered once.  Light edges precede heavy ones in the (w, id) order, so
+// the MSF is unchanged (the argument of P:143 for the two phases).
+// ---------------------------------------------------------------------------
+#ifndef ECL_CROWD_RATIO
+#define ECL_CROWD_RATIO 16   // auto: split when live > this x last round's MSF edges
+#endif
+#ifndef ECL_SPLIT_C
+#define ECL_SPLIT_C 4        // light part: about this many edges per MSF edge of the last round
+#endif
+__device__ __forceinline__ bool crowded(const Params& P, long long live, long long winners, int g) {
+    if (P.refilter == 0 || __ldcg(&P.in->splits) >= 16 || g + 24 >= ECL_MST_MAX_ROUNDS) return false;
+    if (P.refilter > 0) return live > 4 * winners;
+    return live >= (1LL << 20) && live > ECL_CROWD_RATIO * winners;
+}
+
+// T' such that about c = 4 live edges per set (4 x last round's MSF edges,
+// the paper's c = 4 of P:143 applied to the contracted graph) have w < T':
+// every CTA samples its own worklist evenly, then every CTA ranks the same
+// samples (identical result everywhere).  INT_MAX: no useful split.  All
+// threads of all CTAs must call it (one grid barrier).
+__device__ __forceinline__ int split_threshold(const Params& P, const CompactSrc& S, long long live,
+                                               long long winners, cg::grid_group& grid, int* s_w) {
+    const int tid = threadIdx.x;
+    const int ks = max(1, kSplitSamples / P.G);
+    const int ctas = min(P.G, kSplitSampleSlots / ks);   // samples from the first CTAs only
+    if ((int)blockIdx.x < ctas)
+    for (int i = tid; i < ks; i += kBlock) {
+        int w = INT_MAX;   // an empty arena votes "heavy"
+        if (S.cnt > 0) w = __ldcg(&S.base[(long long)(2 * i + 1) * S.cnt / (2 * ks)].z);
+        P.samp[blockIdx.x * ks + i] = w;
+    }
+    grid.sync();
+    const int N = ks * ctas;
+    for (int i = tid; i < N; i += kBlock) s_w[i] = __ldcg(&P.samp[i]);
+    if (tid == 0) s_w[N] = INT_MAX;
+    __syncthreads();
+    long long k = (long long)N * ECL_SPLIT_C * winners / max(live, 1LL);
+    if (k < 1) k = 1;
+    if (k >= N) return INT_MAX;
+    for (int i = tid; i < N; i += kBlock) {
+        const int wi = s_w[i];
+        int less = 0, rank = 0;
+        for (int t = 0; t < N; ++t) {
+            const int wt = s_w[t];
+            less += wt < wi;
+            rank += (wt < wi) || (wt == wi && t < i);
+        }
+        // T' = the sample of rank k, if some sample lies below it (else the
+        // light part could be empty: no split)
+        if (rank == (int)k) s_w[N + 1] = (less > 0 && wi != INT_MAX) ? wi : INT_MAX;
+    }
+    __syncthreads();
+    const int T = s_w[N + 1];
+    __syncthreads();
+    return T;
+}
+
 template <int PH>
 __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
     cg::grid_group grid = cg::this_grid();
-    __shared__ int s_out;
+    __shared__ int s_out, s_def;
     __shared__ long long s_red[3][kWarps];
-    __shared__ int s_pre[kMaxRegionsPerCta + 1];
-    __shared__ int s_rcnt[kMaxRegionsPerCta];
+    // region prefix/counts (first round only) and split samples (later rounds) share one buffer
+    __shared__ int s_buf[kSplitSampleSlots + 2];
+    static_assert(2 * kMaxRegionsPerCta + 1 <= kSplitSampleSlots + 2, "shared buffer");
+    int* const s_pre = s_buf;
+    int* const s_rcnt = s_buf + kMaxRegionsPerCta + 1;
+    int* const s_w = s_buf;
     const int tid = threadIdx.x, lane = tid & 31;
     const bool b0 = blockIdx.x == 0;
     ecl_mst_stats* st = P.st;
@@ -314,13 +398,17 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
     bool overflow = false;
     long long L = __ldcg(&st->live[g]);
     CompactSrc C = compact_src(wl[0], 0);
+    // deferred tuples of a crowded-round split: at the back of this CTA's
+    // arena in buffer hb (-1: none pending), hcnt of them (per CTA; hb is the
+    // same in every CTA because every split decision is)
+    int hb = -1, hcnt = 0;
     // one round: pass B over S, then pass A from S into the other worklist
     auto round = [&](const auto& S) {
         const long long w0 = wcnt;
         passB(P, S, wsum, wcnt);
         const long long d = warp_sum(wcnt - w0);
         if (lane == 0 && d) atomicAdd(reinterpret_cast<unsigned long long*>(&st->winners[g]), (unsigned long long)d);
-        if (tid == 0) s_out = 0;
+        if (tid == 0) s_out = s_def = 0;
         trace_cta(P, 5 + 2 * g);
         grid.sync();
         stamp(P, 5 + 2 * g);
@@ -328,10 +416,55 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
             overflow = true;
             return false;
         }
-        const bool guard = use_guard(P, L, __ldcg(&st->winners[g]));
+        const long long win = __ldcg(&st->winners[g]);
+        const bool guard = use_guard(P, L, win);
         ++g;
-        passA(P, S, wl[cur ^ 1], &s_out, guard);
+        // a split defers to the back of the output arena; with tuples already
+        // deferred (hb >= 0) only when that is the same buffer, below them --
+        // the deferred set is then one run, drained together (any union of
+        // deferred parts is heavier than the light part still running)
+        int T = INT_MAX;
+        if constexpr (std::is_same<std::decay_t<decltype(S)>, CompactSrc>::value) {
+            if ((hb < 0 || hb == (cur ^ 1)) && crowded(P, L, win, g)) {
+                T = split_threshold(P, S, L, win, grid, s_w);
+                if (tid == 0) s_def = hb < 0 ? 0 : hcnt;
+                __syncthreads();
+            }
+        }
+        if (T != INT_MAX) passA<true>(P, S, wl[cur ^ 1], &s_out, guard, T, wl[cur ^ 1] + P.cap, &s_def);
+        else passA(P, S, wl[cur ^ 1], &s_out, guard);
         cur ^= 1;
+        __syncthreads();
+        C = compact_src(wl[cur], s_out);
+        if (T != INT_MAX) {
+            hb = cur;
+            hcnt = s_def;
+            if (b0 && tid == 0) atomicAdd(&P.in->splits, 1);
+        }
+        if (tid == 0 && C.cnt) atomicAdd(reinterpret_cast<unsigned long long*>(&st->live[g]), (unsigned long long)C.cnt);
+        trace_cta(P, 4 + 2 * g);
+        grid.sync();
+        stamp(P, 4 + 2 * g);
+        L = __ldcg(&st->live[g]);
+        return true;
+    };
+    // the light part of a split is done: filter the deferred tuples (find,
+    // drop set(u) == set(v), record, compact) -- a pass A with no pass B
+    // before it, since every key is inf again after the last (empty) round
+    auto drain = [&]() {
+        if (g + 1 >= ECL_MST_MAX_ROUNDS) {
+            overflow = true;
+            return false;
+        }
+        const CompactSrc H = compact_src(wl[hb] + P.cap - hcnt, hcnt);
+        const int ob = hb ^ 1;
+        hb = -1;
+        hcnt = 0;
+        ++g;
+        if (tid == 0) s_out = 0;
+        __syncthreads();
+        passA(P, H, wl[ob], &s_out, true);
+        cur = ob;
         __syncthreads();
         C = compact_src(wl[cur], s_out);
         if (tid == 0 && C.cnt) atomicAdd(reinterpret_cast<unsigned long long*>(&st->live[g]), (unsigned long long)C.cnt);
@@ -341,9 +474,17 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
         L = __ldcg(&st->live[g]);
         return true;
     };
-    if (L > 0 && round(R))
-        while (L > 0 && round(C)) {
+    if (L > 0 && round(R)) {
+        for (;;) {
+            if (L > 0) {
+                if (!round(C)) break;
+            } else if (hb >= 0) {
+                if (!drain()) break;
+            } else {
+                break;
+            }
         }
+    }
     const long long s = warp_sum(wsum), c = warp_sum(wcnt);
     if (lane == 0) {
         if (s) atomicAdd(reinterpret_cast<unsigned long long*>(&st->total_weight), (unsigned long long)s);
@@ -352,6 +493,7 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
     if (b0 && tid == 0) {
         P.in->g_end = g;
         st->rounds = g + 1;
+        st->refilters = __ldcg(&P.in->splits);
         if (overflow) atomicExch(&st->status, ECL_MST_ERR_INPUT);
     }
 }

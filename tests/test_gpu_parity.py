@@ -46,8 +46,9 @@ def assert_parity(m, g, **opts):
 
 
 def check_round_bound(g, stats):
-    """<= ceil(log2 n) + 1 rounds per phase incl. the final empty pass A."""
-    bound = math.ceil(math.log2(max(g.n, 2))) + 1
+    """<= ceil(log2 n) + 1 rounds per phase incl. the final empty pass A; a
+    crowded-round split (opts.refilter) adds one sub-phase of as many."""
+    bound = (math.ceil(math.log2(max(g.n, 2))) + 1) * (1 + stats["refilters"])
     r = stats["rounds"]
     p2 = stats["phase2_round"]
     if p2 < 0:
@@ -96,11 +97,37 @@ def test_config_small(eclmst, name):
     dict(threshold_samples=20), dict(threshold_samples=4096, seed=7),
     dict(populate_order=1), dict(populate_order=2), dict(populate_order=3), dict(populate_order=2, max_ctas=3),
     dict(populate_order=1, max_ctas=2),
+    dict(refilter=0), dict(refilter=1), dict(refilter=1, max_ctas=3), dict(refilter=1, atomic_guards=0),
+    dict(refilter=1, filter=0), dict(refilter=1, path_halving=0, flatten=0),
+    dict(filter_c=2), dict(filter_c=3), dict(filter_c=1, refilter=1), dict(filter_c=64),
 ])
 @pytest.mark.parametrize("name", ["rmat", "uniform", "road"])
 def test_knobs_give_identical_msf(eclmst, name, opts):
     g = synth.make_config(name, "small")
     assert_parity(eclmst, g, **opts)
+
+
+@pytest.mark.parametrize("weights", ["ties", "two", "equal", "uniform"])
+@pytest.mark.parametrize("n,m", [(3000, 60000), (20000, 400000)])
+def test_refilter_forced(eclmst, weights, n, m):
+    """Crowded-round splits (opts.refilter = 1): light part first, deferred
+    part filtered afterwards -- the MSF must not change (P:143 argument)."""
+    g = G.random_small(n, m, seed=n ^ m, weights=weights, multi=True, self_loops=True)
+    stats = assert_parity(eclmst, g, refilter=1)
+    check_round_bound(g, stats)
+    # without the two-phase filter the rounds crowd for sure
+    stats = assert_parity(eclmst, g, refilter=1, filter=0)
+    check_round_bound(g, stats)
+    if weights == "uniform":
+        assert stats["refilters"] >= 1
+
+
+@pytest.mark.parametrize("seed", range(24))
+def test_tiny_adversarial_refilter(eclmst, seed):
+    kinds = ["ties", "equal", "two", "full", "uniform"]
+    g = G.random_small(3 + seed % 13, 10 + (seed * 11) % 90, seed=1000 + seed, weights=kinds[seed % 5],
+                       multi=True, self_loops=seed % 2 == 0)
+    assert_parity(eclmst, g, refilter=1, filter=seed % 3 - 1)
 
 
 def test_two_valued_weights_nontrivial_phase1(eclmst):

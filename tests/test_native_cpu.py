@@ -34,7 +34,7 @@ def test_exports_every_declared_symbol(lib):
 def test_struct_layouts_match_header():
     # header: 8 int32 + 4 int64 + 2 * 128 int64 + 260 int64
     assert ctypes.sizeof(_native.EclMstStats) == 8 * 4 + 4 * 8 + 2 * 128 * 8 + 260 * 8
-    assert ctypes.sizeof(_native.EclMstOptions) == 8 * 4 + 8 + 2 * 4
+    assert ctypes.sizeof(_native.EclMstOptions) == 8 * 4 + 8 + 4 * 4
 
 
 def test_workspace_bytes(lib):
@@ -49,7 +49,7 @@ def test_workspace_bytes(lib):
 def test_argument_validation_without_gpu(lib):
     o = _native.default_options()
     assert o.filter == -1 and o.path_halving == 1 and o.atomic_guards == -1 and o.flatten == 1
-    assert o.seed == 0x5EED and o.threshold_samples == 1024
+    assert o.seed == 0x5EED and o.threshold_samples == 1024 and o.refilter == -1 and o.filter_c == 0
     rc = lib.ecl_mst_device(-1, 0, None, None, None, None, None, None, 0, None, None)
     assert rc == _native.ERR_INVALID
     assert b"negative" in lib.ecl_mst_last_error()
