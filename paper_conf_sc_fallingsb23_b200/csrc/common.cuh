@@ -28,6 +28,7 @@ static_assert(kMaxGrid == ECL_MST_TRACE_CTAS, "trace layout");
 
 struct Internal {
     unsigned long long reps;           // distributed path: sets with a finite key this round
+    long long nroots;                  // distributed path: size of the next round's root list
     unsigned int done;                 // unused ticket
     int g_cur;                         // first global round of the running phase
     int g_end;                         // last global round of the finished phase

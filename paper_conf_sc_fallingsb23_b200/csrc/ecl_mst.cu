@@ -493,7 +493,7 @@ struct DistHandle {
 };
 
 struct DistLayout {
-    size_t stats, internal, rowstart, parent, tgt, keyptrs, shard0, shard_bytes, total;
+    size_t stats, internal, rowstart, parent, tgt, keyptrs, rl0, rl1, rbuf, keep, bcnt, shard0, shard_bytes, total;
     size_t region, acnt, key, wl0, wl1;   // offsets inside one shard block
     long long wl_cap, nlocal_max;
 };
@@ -512,6 +512,11 @@ static inline DistLayout dist_layout(int64_t n, int64_t M, int S, int world) {
     L.parent = off;   off = align_up(off + sizeof(int) * (size_t)n, 256);
     L.tgt = off;      off = align_up(off + sizeof(int) * (size_t)n, 256);
     L.keyptrs = off;  off = align_up(off + sizeof(long long*) * (size_t)S, 256);
+    L.rl0 = off;      off = align_up(off + sizeof(int) * (size_t)n, 256);     // root lists (double buffer)
+    L.rl1 = off;      off = align_up(off + sizeof(int) * (size_t)n, 256);
+    L.rbuf = off;     off = align_up(off + sizeof(long long) * (size_t)n, 256);   // the allreduce buffer
+    L.keep = off;     off = align_up(off + (size_t)n, 256);
+    L.bcnt = off;     off = align_up(off + sizeof(int) * (size_t)kCompactGridMax, 256);
     size_t so = 0;
     L.region = so; so = align_up(so + sizeof(int4) * (size_t)kMaxPopWarps, 256);
     L.acnt = so;   so = align_up(so + sizeof(int) * (size_t)kMaxGrid, 256);
@@ -749,21 +754,40 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
         if ((rc = check("populate"))) return rc;
         bool first = true;
         int cur = 0;
+        // the sets whose keys are exchanged: all n in the phase's first round,
+        // then the roots that can still hold a live edge (root-compacted)
+        const int* R = nullptr;
+        long long nR = n;
+        int rb = 0;
+        int* rl[2] = {reinterpret_cast<int*>(ws + L.rl0), reinterpret_cast<int*>(ws + L.rl1)};
+        long long* rbuf = reinterpret_cast<long long*>(ws + L.rbuf);
+        unsigned char* keep = reinterpret_cast<unsigned char*>(ws + L.keep);
+        int* bcnt = reinterpret_cast<int*>(ws + L.bcnt);
         while (true) {
-            // allreduce(min) of the best-edge keys over all shards
-            if (S > 1) k_vreduce<<<vblocks, 256, 0, s>>>(P0);
-            if ((rc = allreduce(P0.key, (size_t)n, kNcclMin))) return rc;
+            const unsigned rblocks = (unsigned)std::max<long long>(1, std::min<long long>(ceil_div(nR, 256), (long long)di.sms * 8));
+            const unsigned cblocks = (unsigned)std::max<long long>(1, std::min<long long>(ceil_div(nR, 4096), kCompactGridMax));
+            // allreduce(min) of the live sets' best-edge keys over all shards
+            k_dist_gather<<<rblocks, 256, 0, s>>>(P0, R, nR, rbuf);
+            if ((rc = allreduce(rbuf, (size_t)nR, kNcclMin))) return rc;
+            k_dist_scatter<<<rblocks, 256, 0, s>>>(P0, R, nR, rbuf);
             e = cudaMemsetAsync(&in->reps, 0, sizeof(in->reps), s);
             if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "memset: %s", cudaGetErrorString(e));
-            k_dist_reps1<<<vblocks, 256, 0, s>>>(P0);
-            long long reps = 0;
-            if ((rc = read_word(&in->reps, &reps))) return rc;
+            k_dist_reps1<<<rblocks, 256, 0, s>>>(P0, R, nR, rbuf);
+            k_dist_reps2<<<rblocks, 256, 0, s>>>(P0, R, nR, rbuf, keep, g);
+            k_dist_count<<<cblocks, kCompactBlock, 0, s>>>(nR, keep, bcnt);
+            k_dist_compact<<<cblocks, kCompactBlock, 0, s>>>(R, nR, keep, bcnt, rl[rb], &in->nroots);
+            if ((rc = check("rep passes"))) return rc;
+            long long reps = 0, nnext = 0;
+            if ((rc = read_word(&in->reps, &reps))) return rc;   // (syncs; nroots is final too)
+            if ((rc = read_word(&in->nroots, &nnext))) return rc;
             if (reps == 0) {
                 if (first)
                     for (int k = 0; k < S; ++k) k_dist_passA<true><<<sp[k].G, kBlock, 0, s>>>(sp[k], g + 1, cur);
                 break;   // no set has a live edge anywhere: the phase is done
             }
-            k_dist_reps2<<<vblocks, 256, 0, s>>>(P0, g);
+            R = rl[rb];
+            nR = nnext;
+            rb ^= 1;
             if (g + 1 >= ECL_MST_MAX_ROUNDS) return fail(ECL_MST_ERR_INPUT, "round limit");
             ++g;
             for (int k = 0; k < S; ++k) {
