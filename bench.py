@@ -25,6 +25,8 @@ import time
 
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
+# NCCL prints its version banner on stdout at INFO level; rank 0 prints ONE JSON line
+os.environ.setdefault("NCCL_DEBUG", "WARN")
 
 import torch  # noqa: E402
 
