@@ -22,6 +22,7 @@ constexpr int kMaxPopWarps = 65536;            // populate warps (= worklist reg
 constexpr int kMaxRegionsPerCta = 256;         // regions a k_rounds CTA starts from
 constexpr int kTraceSlots = 2 * ECL_MST_MAX_ROUNDS + 4;
 constexpr int kMaxSamples = 4096;              // threshold sample size cap
+constexpr int kStagePieces = 8;                // host path: CSR pieces uploaded under the populate
 constexpr int kSplitSamples = 512;             // crowded-round threshold: about this many samples
 constexpr int kSplitSampleSlots = 1024;        // sample slots (max(1, 512 / G) per CTA, first CTAs)
 static_assert(kMaxGrid == ECL_MST_TRACE_CTAS, "trace layout");
@@ -82,6 +83,7 @@ struct Params {
     int W;                            // populate warps = regions of wl0
     long long rcap;                   // tuples per region
     int pop_contig;                   // bit PH-1: populate<PH> walks contiguous slices of rcap/kChunk chunks
+    int pop_cta0;                     // first populate CTA of this launch (staged host path: pieces)
     const long long* __restrict__ nindex;
     const int* __restrict__ nlist;
     const int* __restrict__ eweight;

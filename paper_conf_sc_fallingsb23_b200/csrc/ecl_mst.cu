@@ -138,10 +138,41 @@ size_t ecl_mst_workspace_bytes(int64_t n, int64_t M) {
     return layout_for(n, M).total;
 }
 
+}  // extern "C"
+
+namespace eclmst {
+// The host path's staged upload (NEXT-1, the paper's memcpy variant P:325):
+// the CSR arrives on a copy stream in pieces, each piece the CSR range of one
+// group of populate CTAs (contiguous slices), and each group's populate starts
+// as soon as its piece has landed, so the populate hides under the PCIe copy.
+struct Staging {
+    cudaStream_t copy;                 // copy stream (the compute stream is the call's)
+    const int64_t* h_idx;              // host CSR (pinned for overlap)
+    const int32_t* h_list;
+    const int32_t* h_w;
+    cudaEvent_t ev[kStagePieces + 2];  // [0]: nindex (+ eweight when sampled), [1 + k]: piece k
+};
+}  // namespace eclmst
+
+static int run_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t* nlist, const int32_t* eweight,
+                      uint8_t* in_mst_out, int64_t* total_weight_out, void* workspace, size_t workspace_bytes,
+                      const ecl_mst_options* opts, void* stream, const Staging* stg);
+
+extern "C" {
+
 int ecl_mst_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t* nlist, const int32_t* eweight,
                    uint8_t* in_mst_out, int64_t* total_weight_out, void* workspace, size_t workspace_bytes,
                    const ecl_mst_options* opts, void* stream) {
     g_last_error.clear();
+    return run_device(n, M, nindex, nlist, eweight, in_mst_out, total_weight_out, workspace, workspace_bytes, opts,
+                      stream, nullptr);
+}
+
+}  // extern "C"
+
+static int run_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t* nlist, const int32_t* eweight,
+                      uint8_t* in_mst_out, int64_t* total_weight_out, void* workspace, size_t workspace_bytes,
+                      const ecl_mst_options* opts, void* stream, const Staging* stg) {
     if (n < 0 || M < 0) return fail(ECL_MST_ERR_INVALID, "negative n or M");
     if (M > (int64_t)0xFFFFFFFFLL) return fail(ECL_MST_ERR_TOO_LARGE, "M = %lld exceeds 2^32-1", (long long)M);
     if (!total_weight_out || !workspace) return fail(ECL_MST_ERR_INVALID, "null total_weight_out or workspace");
@@ -210,6 +241,7 @@ int ecl_mst_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t* n
     P.W = (int)W;
     P.rcap = rcap;
     P.pop_contig = contig;
+    P.pop_cta0 = 0;
     P.nindex = reinterpret_cast<const long long*>(nindex);
     P.nlist = nlist;
     P.eweight = eweight;
@@ -268,7 +300,40 @@ int ecl_mst_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t* n
         return timing ? cudaEventRecord(g_timing.ev[ev_i++], s) : cudaSuccess;
     };
     const unsigned flat_blocks = (unsigned)std::max<long long>(init_blocks, 1);
-    cudaError_t e = mark();
+    // staged upload: CTA groups of the phase-1 populate and their CSR pieces
+    const bool staged = stg && (contig & 1);
+    const int pieces = staged ? (int)std::min<long long>(kStagePieces, pop_blocks) : 1;
+    auto group_cta = [&](int k) { return (long long)(pop_blocks * k / pieces); };
+    cudaError_t e = cudaSuccess;
+    if (stg) {
+        // nindex first (k_init needs all of it), and eweight too when the
+        // threshold samples it; then the pieces of nlist (and eweight)
+        const bool sampled = (P.filter_mode > 0 || (P.filter_mode < 0 && M >= 4LL * n)) && P.threshold_mode == 0;
+        e = cudaMemcpyAsync(const_cast<int64_t*>(nindex), stg->h_idx, sizeof(int64_t) * ((size_t)n + 1),
+                            cudaMemcpyHostToDevice, stg->copy);
+        if (e == cudaSuccess && sampled)
+            e = cudaMemcpyAsync(const_cast<int32_t*>(eweight), stg->h_w, sizeof(int32_t) * (size_t)M,
+                                cudaMemcpyHostToDevice, stg->copy);
+        if (e == cudaSuccess) e = cudaEventRecord(stg->ev[0], stg->copy);
+        const long long span = rcap / kChunk;
+        for (int k = 0; k < pieces && e == cudaSuccess; ++k) {
+            long long e0 = staged ? std::min<long long>(M, group_cta(k) * kPopWarps * span * kChunk) : 0;
+            long long e1 = staged ? std::min<long long>(M, group_cta(k + 1) * kPopWarps * span * kChunk) : M;
+            if (k == pieces - 1) e1 = M;
+            if (e1 > e0) {
+                e = cudaMemcpyAsync(const_cast<int32_t*>(nlist) + e0, stg->h_list + e0, sizeof(int32_t) * (size_t)(e1 - e0),
+                                    cudaMemcpyHostToDevice, stg->copy);
+                if (e == cudaSuccess && !sampled)
+                    e = cudaMemcpyAsync(const_cast<int32_t*>(eweight) + e0, stg->h_w + e0,
+                                        sizeof(int32_t) * (size_t)(e1 - e0), cudaMemcpyHostToDevice, stg->copy);
+            }
+            if (e == cudaSuccess) e = cudaEventRecord(stg->ev[1 + k], stg->copy);
+        }
+        if (e == cudaSuccess) e = cudaStreamWaitEvent(s, stg->ev[0], 0);
+        if (e == cudaSuccess && !staged) e = cudaStreamWaitEvent(s, stg->ev[1], 0);
+        if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "staged H2D: %s", cudaGetErrorString(e));
+    }
+    if (e == cudaSuccess) e = mark();
     if (e == cudaSuccess) e = cudaMemsetAsync(P.st, 0, sizeof(ecl_mst_stats), s);
     if (e == cudaSuccess) {
         k_init<<<flat_blocks, 256, 0, s>>>(P);
@@ -276,8 +341,22 @@ int ecl_mst_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t* n
     }
     if (e == cudaSuccess) e = mark();
     if (e == cudaSuccess) {
-        k_populate<1><<<(unsigned)pop_blocks, kPopBlock, 0, s>>>(P);
-        e = cudaGetLastError();
+        if (staged) {   // one launch per piece, each after its piece has landed
+            for (int k = 0; k < pieces && e == cudaSuccess; ++k) {
+                const long long c0 = group_cta(k), c1 = group_cta(k + 1);
+                if (c1 <= c0) continue;
+                e = cudaStreamWaitEvent(s, stg->ev[1 + k], 0);
+                Params Pk = P;
+                Pk.pop_cta0 = (int)c0;
+                if (e == cudaSuccess) {
+                    k_populate<1><<<(unsigned)(c1 - c0), kPopBlock, 0, s>>>(Pk);
+                    e = cudaGetLastError();
+                }
+            }
+        } else {
+            k_populate<1><<<(unsigned)pop_blocks, kPopBlock, 0, s>>>(P);
+            e = cudaGetLastError();
+        }
     }
     if (e == cudaSuccess) e = mark();
     if (e == cudaSuccess)
@@ -310,6 +389,8 @@ int ecl_mst_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t* n
     if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "launch (G=%lld): %s", G, cudaGetErrorString(e));
     return ECL_MST_OK;
 }
+
+extern "C" {
 
 int ecl_mst_kernel_times(float* ms_out, int32_t max_stages) {
     g_last_error.clear();
@@ -353,14 +434,22 @@ static void* g_pool = nullptr;
 static size_t g_pool_cap = 0;
 static int g_pool_dev = -1;
 static cudaStream_t g_pool_stream = nullptr;
+static cudaStream_t g_pool_copy = nullptr;          // staged upload (NEXT-1)
+static cudaEvent_t g_pool_ev[kStagePieces + 2];
+static bool g_pool_ev_ok = false;
 
 void ecl_mst_release_host_cache(void) {
     std::lock_guard<std::mutex> lk(g_pool_mu);
     if (g_pool) cudaFree(g_pool);
     if (g_pool_stream) cudaStreamDestroy(g_pool_stream);
+    if (g_pool_copy) cudaStreamDestroy(g_pool_copy);
+    if (g_pool_ev_ok)
+        for (auto& ev : g_pool_ev) cudaEventDestroy(ev);
     g_pool = nullptr;
     g_pool_cap = 0;
     g_pool_stream = nullptr;
+    g_pool_copy = nullptr;
+    g_pool_ev_ok = false;
     g_pool_dev = -1;
 }
 
@@ -400,6 +489,11 @@ int64_t ecl_mst(int32_t n, const int64_t* nindex, const int32_t* nlist, const in
         if (g_pool_stream && g_pool_dev != dev) {
             cudaStreamDestroy(g_pool_stream);
             g_pool_stream = nullptr;
+            if (g_pool_copy) cudaStreamDestroy(g_pool_copy);
+            g_pool_copy = nullptr;
+            if (g_pool_ev_ok)
+                for (auto& ev : g_pool_ev) cudaEventDestroy(ev);
+            g_pool_ev_ok = false;
         }
         e = cudaMalloc(&g_pool, need);
         if (e == cudaSuccess) {
@@ -408,6 +502,15 @@ int64_t ecl_mst(int32_t n, const int64_t* nindex, const int32_t* nlist, const in
         }
     }
     if (e == cudaSuccess && !g_pool_stream) e = cudaStreamCreateWithFlags(&g_pool_stream, cudaStreamNonBlocking);
+    if (e == cudaSuccess && !g_pool_copy) e = cudaStreamCreateWithFlags(&g_pool_copy, cudaStreamNonBlocking);
+    if (e == cudaSuccess && !g_pool_ev_ok) {
+        int made = 0;
+        for (; made < kStagePieces + 2 && e == cudaSuccess; ++made)
+            e = cudaEventCreateWithFlags(&g_pool_ev[made], cudaEventDisableTiming);
+        if (e == cudaSuccess) g_pool_ev_ok = true;
+        else
+            for (int i = 0; i + 1 < made; ++i) cudaEventDestroy(g_pool_ev[i]);
+    }
     if (e != cudaSuccess) {
         fail(ECL_MST_ERR_CUDA, "host path setup: %s", cudaGetErrorString(e));
         return INT64_MIN;
@@ -420,15 +523,19 @@ int64_t ecl_mst(int32_t n, const int64_t* nindex, const int32_t* nlist, const in
     int64_t* d_tot = reinterpret_cast<int64_t*>(base + b_idx + 2 * b_list + b_mst);
     void* d_ws = base + b_idx + 2 * b_list + b_mst + b_tot;
     cudaStream_t s = g_pool_stream;
-    e = cudaMemcpyAsync(d_idx, nindex, sizeof(int64_t) * ((size_t)n + 1), cudaMemcpyHostToDevice, s);
-    if (e == cudaSuccess) e = cudaMemcpyAsync(d_list, nlist, sizeof(int32_t) * (size_t)M, cudaMemcpyHostToDevice, s);
-    if (e == cudaSuccess) e = cudaMemcpyAsync(d_w, eweight, sizeof(int32_t) * (size_t)M, cudaMemcpyHostToDevice, s);
-    if (e != cudaSuccess) {
-        fail(ECL_MST_ERR_CUDA, "H2D: %s", cudaGetErrorString(e));
+    // H2D on the copy stream in pieces; each piece's populate starts when it lands
+    Staging stg;
+    stg.copy = g_pool_copy;
+    stg.h_idx = nindex;
+    stg.h_list = nlist;
+    stg.h_w = eweight;
+    for (int i = 0; i < kStagePieces + 2; ++i) stg.ev[i] = g_pool_ev[i];
+    int rc = run_device(n, M, d_idx, d_list, d_w, d_mst, d_tot, d_ws, b_ws, nullptr, s, &stg);
+    if (rc) {
+        cudaStreamSynchronize(g_pool_copy);   // no copy may outlive the caller's buffers
+        cudaStreamSynchronize(s);
         return INT64_MIN;
     }
-    int rc = ecl_mst_device(n, M, d_idx, d_list, d_w, d_mst, d_tot, d_ws, b_ws, nullptr, s);
-    if (rc) return INT64_MIN;
     int64_t total = INT64_MIN;
     e = cudaMemcpyAsync(in_mst_out, d_mst, (size_t)M, cudaMemcpyDeviceToHost, s);
     if (e == cudaSuccess) e = cudaMemcpyAsync(&total, d_tot, sizeof total, cudaMemcpyDeviceToHost, s);

@@ -107,7 +107,7 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
     // every region -- and every k_rounds CTA -- gets the same mix even where
     // the density of u < v entries drifts along the rows) and appends its
     // tuples densely to its own region: no atomics, no CTA barrier.
-    const int w = blockIdx.x * kPopWarps + warp;
+    const int w = (P.pop_cta0 + (int)blockIdx.x) * kPopWarps + warp;
     if (w >= P.W) return;   // (sharded path: partial last CTA)
     int4* const out = P.wl0 + (long long)w * P.rcap;
     int cnt = 0, canon_cnt = 0, heavy_cnt = 0;

@@ -185,6 +185,24 @@ def test_deterministic_and_reusable_workspace(eclmst):
         assert torch.equal(a, b) and int(tb.item()) == ta
 
 
+@pytest.mark.parametrize("name", ["grid", "rmat", "uniform", "rgg"])
+def test_host_api_staged_upload(eclmst, name):
+    """The host path uploads the CSR in pieces under the populate (NEXT-1):
+    same MSF as the oracle for filtered (eweight sampled first) and
+    unfiltered graphs, pinned and pageable host buffers."""
+    g = synth.make_config(name, "small")
+    omask, ototal, _ = oracle.kruskal_graph(g)
+    for pin in (True, False):
+        out = torch.empty(g.M, dtype=torch.uint8)
+        args = (g.nindex, g.nlist, g.eweight)
+        if pin:
+            out = out.pin_memory()
+            args = tuple(a.pin_memory() for a in args)
+        total = eclmst.ecl_mst(g.n, *args, out)
+        assert total == ototal
+        assert np.array_equal(out.numpy(), omask)
+
+
 def test_host_api_memcpy_variant(eclmst):
     g = synth.make_config("road", "small")
     omask, ototal, _ = oracle.kruskal_graph(g)
