@@ -81,7 +81,7 @@ typedef struct ecl_mst_options {
                                 P:152) to the live worklist -- edges below a sampled threshold T'
                                 run to completion first, the rest are deferred and filtered by
                                 set(u) != set(v) afterwards.  -1 (default) auto: when >= 2^20 live
-                                tuples and > 16 per MSF edge of the last round; 0 never; 1 whenever
+                                tuples and > 6 per MSF edge of the last round; 0 never; 1 whenever
                                 live > 4 x last round's MSF edges (tests).  Same MSF either way. */
     int32_t filter_c;        /* c of P:143: the threshold targets the c|V| lightest CSR entries.
                                 0 (default) = 4, "we use c = 4 in our code"; P:394 aims
