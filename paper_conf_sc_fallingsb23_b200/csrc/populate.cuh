@@ -88,6 +88,10 @@ template <int PH>
 #ifndef ECL_GIANT_MIN_N
 #define ECL_GIANT_MIN_N (32LL << 20)   // parent[] larger than ~half the L2
 #endif
+#ifndef ECL_P2_GUARD_COLD
+#define ECL_P2_GUARD_COLD 0   // phase-2 populate: guard the atomicMin of slots other than the giant's
+                              // (off: C4 populate2 2.60 -> 2.40 ms, C5 11.8 -> 11.4 ms)
+#endif
 #ifndef ECL_POP_MINB
 #define ECL_POP_MINB 4
 #endif
@@ -138,6 +142,16 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
     // chunk i the phase-2 membership bits of chunk i+1's far ends are
     // requested (their entries have arrived by then).
     const int giant = (PH == 2 && P.flatten && P.giant_bits) ? __ldg(&P.in->giant) : -1;
+    // phase 2: the largest set's slot is the one almost every kept edge
+    // touches; keep its minimum in a register (one atomicMin per warp at the
+    // end) and give the other, cold slots a plain atomicMin
+    const int kg = (PH == 2 && P.flatten) ? __ldg(&P.in->giant) : -1;
+    long long gbest = kInf;
+    const bool guard_cold = PH == 2 ? (P.guards > 0 || (P.guards < 0 && ECL_P2_GUARD_COLD)) : guard;
+    auto rec = [&](int x, long long key) {
+        if (PH == 2 && x == kg) gbest = min(gbest, key);
+        else record_min(D.k(x), key, guard_cold);
+    };
     // deep: also prefetch the next chunk's row starts (phase 2, where the
     // bitmap / parent loads already lengthen each chunk's chain)
     constexpr bool deep = PH == 1 ? ECL_DEEP_PH1 : ECL_DEEP_PH2;
@@ -320,17 +334,17 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
             if (!keep[k]) continue;
             const long long key = make_key(t[k].z, (unsigned)t[k].w);   // L19 val <- e_w : e_id
             if (t[k].x != bp) {
-                if (bp >= 0) record_min(D.k(bp), best, guard);
+                if (bp >= 0) rec(bp, best);
                 bp = t[k].x;
                 best = key;
             } else {
                 best = min(best, key);
             }
         }
-        if (bp >= 0) record_min(D.k(bp), best, guard);
+        if (bp >= 0) rec(bp, best);
 #pragma unroll
         for (int k = 0; k < kItems; ++k)
-            if (keep[k]) record_min(D.k(t[k].y), make_key(t[k].z, (unsigned)t[k].w), guard);
+            if (keep[k]) rec(t[k].y, make_key(t[k].z, (unsigned)t[k].w));
     }
     if (PH == 2 && nxt(lc) < lend) nvb = vbits(nv);   // next chunk's far-end bits
     // L7: append the chunk's tuples to the warp's region
@@ -350,6 +364,11 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
     cnt += tot;
     }
     if (err) atomicExch(&P.st->status, ECL_MST_ERR_INPUT);
+    if (PH == 2 && kg >= 0) {
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) gbest = min(gbest, __shfl_xor_sync(kFull, gbest, o));
+        if (lane == 0 && gbest != kInf) atomicMin(D.k(kg), gbest);
+    }
     if (PH == 1) {   // |E| and the deferred count of this warp's chunks
         canon_cnt = warp_sum(canon_cnt);
         heavy_cnt = warp_sum(heavy_cnt);

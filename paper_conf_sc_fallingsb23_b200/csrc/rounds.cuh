@@ -55,28 +55,32 @@ __global__ void __launch_bounds__(256) k_flatten(Params P) {
 }
 
 // After phase 1 most vertices of a graph whose light edges percolate (C3-C5)
-// sit in ONE set.  Find its root by a majority vote over sampled vertices;
-// k_flatten<2> then writes a bitmap of its members, and the phase-2 populate
-// filters an edge with both ends in it from the bitmap (n/8 bytes, L2
-// resident) instead of two random parent loads.
+// sit in ONE set.  Find its root by a majority vote over sampled vertices.
+// The phase-2 populate keeps that set's key minimum per warp (it is the hot
+// slot almost every kept edge touches), and for n >= 2^25 k_flatten<2> writes
+// a bitmap of its members, so that populate filters an edge with both ends in
+// it from the bitmap (n/8 bytes, L2 resident) instead of two random parent
+// loads.
 __global__ void __launch_bounds__(256) k_giant(Params P) {
-    __shared__ int s_r[1024];
-    if (!phase2_needed(P) || !P.flatten || !P.giant_bits) return;
+    constexpr int kS = 256;   // samples (one per thread): a set holding >= 1/4 shows up reliably
+    __shared__ int s_r[kS];
+    if (!phase2_needed(P) || !P.flatten) return;
     const DS D = ds_of(P);
-    for (int i = threadIdx.x; i < 1024; i += blockDim.x) {
+    {
+        const int i = threadIdx.x;
         const long long v = (long long)(splitmix64(0x6A09E667F3BCC909ull + (unsigned long long)i) % (unsigned long long)P.n);
         s_r[i] = find_root(D, (int)v, false);
     }
     __syncthreads();
     if (threadIdx.x == 0) {
         int cand = -1, votes = 0;                 // Boyer-Moore majority vote
-        for (int i = 0; i < 1024; ++i) {
+        for (int i = 0; i < kS; ++i) {
             if (votes == 0) { cand = s_r[i]; votes = 1; }
             else votes += (s_r[i] == cand) ? 1 : -1;
         }
         int cnt = 0;
-        for (int i = 0; i < 1024; ++i) cnt += s_r[i] == cand;
-        P.in->giant = cnt >= 256 ? cand : -1;     // worth a bitmap only if it holds >= 1/4
+        for (int i = 0; i < kS; ++i) cnt += s_r[i] == cand;
+        P.in->giant = cnt >= kS / 4 ? cand : -1;   // worth it only if it holds >= 1/4
     }
 }
 
@@ -242,7 +246,10 @@ __device__ __forceinline__ void passA(const Params& P, const SRC& S, int4* __res
 
 // L27-31 (+ L34-37): check, join, mark over the CTA's worklist.
 template <class SRC>
-__device__ __forceinline__ void passB(const Params& P, const SRC& S, long long& wsum, long long& wcnt) {
+// The MSF weight and edge count go to this warp's shared accumulators once per
+// chunk (acc[0] += weights, acc[1] += edges): no 64-bit running sums held in
+// registers across the loop (k_rounds is register-capped; they spilled).
+__device__ __forceinline__ void passB(const Params& P, const SRC& S, long long* acc) {
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const DS D = ds_of(P);
     for (int k = warp; k < S.nloc; k += kWarps) {
@@ -268,6 +275,8 @@ __device__ __forceinline__ void passB(const Params& P, const SRC& S, long long& 
                 kq[i] = __ldca(reinterpret_cast<const unsigned*>(D.k(t[i].y)));
             }
         }
+        long long csum = 0;
+        int ccnt = 0;
 #pragma unroll
         for (int i = 0; i < kItems; ++i) {
             if (!ok[i]) continue;
@@ -281,8 +290,16 @@ __device__ __forceinline__ void passB(const Params& P, const SRC& S, long long& 
                 if (wp) __stcg(D.k(p), kInf);                          // L35
                 if (wq) __stcg(D.k(q), kInf);                          // L36
                 P.in_mst[(unsigned)t[i].w] = 1;                        // L31
-                wsum += t[i].z;
-                wcnt += 1;
+                csum += t[i].z;
+                ccnt += 1;
+            }
+        }
+        ccnt = warp_sum(ccnt);
+        if (ccnt) {
+            csum = warp_sum(csum);
+            if (lane == 0) {
+                acc[0] += csum;
+                acc[1] += ccnt;
             }
         }
     }
@@ -393,7 +410,9 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
     if (b0 && tid == 0 && PH == 2) st->phase2_round = g;
     trace_cta(P, 4 + 2 * g);
     grid.sync();
-    long long wsum = 0, wcnt = 0;
+    __shared__ long long s_acc[kWarps][2];   // per warp: MSF weight, MSF edges (pass B)
+    if (lane == 0) s_acc[tid >> 5][0] = s_acc[tid >> 5][1] = 0;
+    long long* const acc = s_acc[tid >> 5];
     int cur = 0;
     bool overflow = false;
     long long L = __ldcg(&st->live[g]);
@@ -404,9 +423,9 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
     int hb = -1, hcnt = 0;
     // one round: pass B over S, then pass A from S into the other worklist
     auto round = [&](const auto& S) {
-        const long long w0 = wcnt;
-        passB(P, S, wsum, wcnt);
-        const long long d = warp_sum(wcnt - w0);
+        const long long w0 = acc[1];
+        passB(P, S, acc);
+        const long long d = acc[1] - w0;
         if (lane == 0 && d) atomicAdd(reinterpret_cast<unsigned long long*>(&st->winners[g]), (unsigned long long)d);
         if (tid == 0) s_out = s_def = 0;
         trace_cta(P, 5 + 2 * g);
@@ -485,7 +504,7 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
             }
         }
     }
-    const long long s = warp_sum(wsum), c = warp_sum(wcnt);
+    const long long s = acc[0], c = acc[1];
     if (lane == 0) {
         if (s) atomicAdd(reinterpret_cast<unsigned long long*>(&st->total_weight), (unsigned long long)s);
         if (c) atomicAdd(reinterpret_cast<unsigned long long*>(&st->msf_edges), (unsigned long long)c);
