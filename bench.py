@@ -25,8 +25,19 @@ import time
 
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
-# NCCL prints its version banner on stdout at INFO level; rank 0 prints ONE JSON line
+# Rank 0 prints ONE JSON line on stdout.  Native libraries (NCCL prints a
+# version banner at NCCL_DEBUG >= VERSION, which includes WARN) write to fd 1
+# directly, so fd 1 is pointed at stderr for the whole run and the JSON line
+# goes to a private duplicate of the original stdout.
 os.environ.setdefault("NCCL_DEBUG", "WARN")
+_JSON_OUT = os.fdopen(os.dup(1), "w")
+os.dup2(2, 1)
+
+
+def emit(line):
+    _JSON_OUT.write(json.dumps(line) + "\n")
+    _JSON_OUT.flush()
+
 
 import torch  # noqa: E402
 
@@ -254,7 +265,7 @@ def run_reference(args, rank, world):
                          "sample": f"whole {g.name} graph per step (serial C Kruskal, oracle/kruskal.c)"},
         "e2e": {"value": value, "unit": "edges/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
-    print(json.dumps(line), flush=True)
+    emit(line)
 
 
 def main():
@@ -489,7 +500,7 @@ def main():
                   "stage_us": None if use_dist else stage_times(st)},
         "gen_s": t_gen,
     }
-    print(json.dumps(line), flush=True)
+    emit(line)
     if use_dist:
         eclmst.ecl_mst_dist_finalize(handle)
         torch.distributed.destroy_process_group()

@@ -146,15 +146,29 @@ __global__ void __launch_bounds__(kCompactBlock) k_dist_count(long long nR, cons
     }
 }
 
+// The last block also publishes {sets with a finite key, |R_next|} to a
+// mapped pinned host word pair (host_out, may be null) -- the host loop reads
+// them after an event on this kernel while the next pass A already runs --
+// and zeroes the set counter for the next round.
 __global__ void __launch_bounds__(kCompactBlock) k_dist_compact(const int* R, long long nR, const unsigned char* keep,
-                                                                const int* bcnt, int* Rnext, long long* nnext) {
+                                                                const int* bcnt, int* Rnext, long long* nnext,
+                                                                unsigned long long* reps,
+                                                                volatile long long* host_out) {
     __shared__ int s_base, s_w[kCompactBlock / 32];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     if (threadIdx.x == 0) {
         int b = 0;
         for (unsigned k = 0; k < blockIdx.x; ++k) b += bcnt[k];
         s_base = b;
-        if (blockIdx.x == gridDim.x - 1) *nnext = (long long)b + bcnt[blockIdx.x];
+        if (blockIdx.x == gridDim.x - 1) {
+            const long long nn = (long long)b + bcnt[blockIdx.x];
+            *nnext = nn;
+            if (host_out) {
+                host_out[0] = (long long)*reps;
+                host_out[1] = nn;
+            }
+            *reps = 0;
+        }
     }
     __syncthreads();
     long long lo, hi;

@@ -596,8 +596,18 @@ static int load_nccl() {
 struct DistHandle {
     int rank = 0, world = 1;
     NcclComm comm = nullptr;
-    long long* h_pin = nullptr;   // pinned host word for the per-round set count
+    long long* h_pin = nullptr;   // pinned host words (phase-2 decision, stats)
+    long long* h_map = nullptr;   // mapped pinned pair {sets with a finite key, |R_next|}, written by k_dist_compact
+    long long* d_map = nullptr;   // its device alias
+    cudaEvent_t ev = nullptr;     // recorded after k_dist_compact each round
 };
+
+static void release(DistHandle* h) {
+    if (h->ev) cudaEventDestroy(h->ev);
+    if (h->h_map) cudaFreeHost(h->h_map);
+    if (h->h_pin) cudaFreeHost(h->h_pin);
+    delete h;
+}
 
 struct DistLayout {
     size_t stats, internal, rowstart, parent, tgt, keyptrs, rl0, rl1, rbuf, keep, bcnt, shard0, shard_bytes, total;
@@ -658,14 +668,17 @@ int ecl_mst_dist_init(const void* uid, int32_t rank, int32_t world, void** handl
     h->rank = rank;
     h->world = world;
     cudaError_t e = cudaHostAlloc(reinterpret_cast<void**>(&h->h_pin), sizeof(long long) * 4, cudaHostAllocDefault);
+    if (e == cudaSuccess)
+        e = cudaHostAlloc(reinterpret_cast<void**>(&h->h_map), sizeof(long long) * 2, cudaHostAllocMapped);
+    if (e == cudaSuccess) e = cudaHostGetDevicePointer(reinterpret_cast<void**>(&h->d_map), h->h_map, 0);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->ev, cudaEventDisableTiming);
     if (e != cudaSuccess) {
-        delete h;
-        return fail(ECL_MST_ERR_CUDA, "cudaHostAlloc: %s", cudaGetErrorString(e));
+        release(h);
+        return fail(ECL_MST_ERR_CUDA, "dist_init: %s", cudaGetErrorString(e));
     }
     if (world > 1 || uid) {   // world 1 with a uid: a one-rank NCCL communicator (tests the NCCL path)
         if (!uid) {
-            cudaFreeHost(h->h_pin);
-            delete h;
+            release(h);
             return fail(ECL_MST_ERR_INVALID, "world > 1 needs an NCCL unique id");
         }
         int rc = load_nccl();
@@ -676,8 +689,7 @@ int ecl_mst_dist_init(const void* uid, int32_t rank, int32_t world, void** handl
             if (r) rc = fail(ECL_MST_ERR_CUDA, "ncclCommInitRank: %s", g_nccl.getErrorString ? g_nccl.getErrorString(r) : "?");
         }
         if (rc) {
-            cudaFreeHost(h->h_pin);
-            delete h;
+            release(h);
             return rc;
         }
     }
@@ -690,8 +702,7 @@ int ecl_mst_dist_finalize(void* handle) {
     DistHandle* h = static_cast<DistHandle*>(handle);
     if (!h) return ECL_MST_OK;
     if (h->comm && g_nccl.ok) g_nccl.commDestroy(h->comm);
-    if (h->h_pin) cudaFreeHost(h->h_pin);
-    delete h;
+    release(h);
     return ECL_MST_OK;
 }
 
@@ -833,6 +844,7 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
     };
 
     if (e == cudaSuccess) e = cudaMemsetAsync(st, 0, sizeof(ecl_mst_stats), s);
+    if (e == cudaSuccess) e = cudaMemsetAsync(in, 0, sizeof(Internal), s);   // (reps: zeroed again by each k_dist_compact)
     if (e == cudaSuccess) e = cudaMemsetAsync(in_mst_out, 0, (size_t)M, s);   // every rank returns the full mask
     if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "memset: %s", cudaGetErrorString(e));
     k_init<<<vblocks, 256, 0, s>>>(P0);
@@ -870,40 +882,58 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
         long long* rbuf = reinterpret_cast<long long*>(ws + L.rbuf);
         unsigned char* keep = reinterpret_cast<unsigned char*>(ws + L.keep);
         int* bcnt = reinterpret_cast<int*>(ws + L.bcnt);
+        // Each round is enqueued in full -- exchange, rep passes, root-list
+        // compaction, and the next pass A -- before the host waits, on an
+        // event behind the compaction, for the two words that decide the next
+        // round (its root-list size, and whether any set still had a live
+        // edge).  The pass A is speculative: when no set had a live edge every
+        // worklist is already empty and it records nothing.  So the GPU runs
+        // that pass A while the host reads the counts and enqueues the next
+        // exchange: no stream drain per round.
         while (true) {
             const unsigned rblocks = (unsigned)std::max<long long>(1, std::min<long long>(ceil_div(nR, 256), (long long)di.sms * 8));
             const unsigned cblocks = (unsigned)std::max<long long>(1, std::min<long long>(ceil_div(nR, 4096), kCompactGridMax));
-            // allreduce(min) of the live sets' best-edge keys over all shards
-            k_dist_gather<<<rblocks, 256, 0, s>>>(P0, R, nR, rbuf);
-            if ((rc = allreduce(rbuf, (size_t)nR, kNcclMin))) return rc;
-            k_dist_scatter<<<rblocks, 256, 0, s>>>(P0, R, nR, rbuf);
-            e = cudaMemsetAsync(&in->reps, 0, sizeof(in->reps), s);
-            if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "memset: %s", cudaGetErrorString(e));
-            k_dist_reps1<<<rblocks, 256, 0, s>>>(P0, R, nR, rbuf);
-            k_dist_reps2<<<rblocks, 256, 0, s>>>(P0, R, nR, rbuf, keep, g);
-            k_dist_count<<<cblocks, kCompactBlock, 0, s>>>(nR, keep, bcnt);
-            k_dist_compact<<<cblocks, kCompactBlock, 0, s>>>(R, nR, keep, bcnt, rl[rb], &in->nroots);
-            if ((rc = check("rep passes"))) return rc;
-            long long reps = 0, nnext = 0;
-            if ((rc = read_word(&in->reps, &reps))) return rc;   // (syncs; nroots is final too)
-            if ((rc = read_word(&in->nroots, &nnext))) return rc;
-            if (reps == 0) {
-                if (first)
-                    for (int k = 0; k < S; ++k) k_dist_passA<true><<<sp[k].G, kBlock, 0, s>>>(sp[k], g + 1, cur);
-                break;   // no set has a live edge anywhere: the phase is done
+            // allreduce(min) of the live sets' best-edge keys over all shards.
+            // A phase's first round exchanges all n keys: with one local shard
+            // that is key[] itself, reduced in place (no gather/scatter copies;
+            // reps2 resets key[x] only after reading it as buf[x]).
+            long long* xbuf = rbuf;
+            if (R == nullptr && S == 1) {
+                xbuf = P0.key;
+                if ((rc = allreduce(xbuf, (size_t)nR, kNcclMin))) return rc;
+            } else {
+                k_dist_gather<<<rblocks, 256, 0, s>>>(P0, R, nR, rbuf);
+                if ((rc = allreduce(rbuf, (size_t)nR, kNcclMin))) return rc;
+                k_dist_scatter<<<rblocks, 256, 0, s>>>(P0, R, nR, rbuf);
             }
+            k_dist_reps1<<<rblocks, 256, 0, s>>>(P0, R, nR, xbuf);
+            k_dist_reps2<<<rblocks, 256, 0, s>>>(P0, R, nR, xbuf, keep, g);
+            k_dist_count<<<cblocks, kCompactBlock, 0, s>>>(nR, keep, bcnt);
+            k_dist_compact<<<cblocks, kCompactBlock, 0, s>>>(R, nR, keep, bcnt, rl[rb], &in->nroots, &in->reps, h->d_map);
+            e = cudaEventRecord(h->ev, s);
+            if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "event: %s", cudaGetErrorString(e));
+            const bool can_continue = g + 1 < ECL_MST_MAX_ROUNDS;
+            if (can_continue) {
+                // (first: also counts the phase's populate output -- needed even
+                // when the phase turns out empty)
+                for (int k = 0; k < S; ++k) {
+                    if (first) k_dist_passA<true><<<sp[k].G, kBlock, 0, s>>>(sp[k], g + 1, cur);
+                    else k_dist_passA<false><<<sp[k].G, kBlock, 0, s>>>(sp[k], g + 1, cur);
+                }
+            }
+            if ((rc = check("rounds"))) return rc;
+            e = cudaEventSynchronize(h->ev);
+            if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "sync: %s", cudaGetErrorString(e));
+            const long long reps = reinterpret_cast<volatile long long*>(h->h_map)[0];
+            const long long nnext = reinterpret_cast<volatile long long*>(h->h_map)[1];
+            if (reps == 0) break;   // no set has a live edge anywhere: the phase is done
+            if (!can_continue) return fail(ECL_MST_ERR_INPUT, "round limit");
             R = rl[rb];
             nR = nnext;
             rb ^= 1;
-            if (g + 1 >= ECL_MST_MAX_ROUNDS) return fail(ECL_MST_ERR_INPUT, "round limit");
             ++g;
-            for (int k = 0; k < S; ++k) {
-                if (first) k_dist_passA<true><<<sp[k].G, kBlock, 0, s>>>(sp[k], g, cur);
-                else k_dist_passA<false><<<sp[k].G, kBlock, 0, s>>>(sp[k], g, cur);
-            }
             cur ^= 1;
             first = false;
-            if ((rc = check("rounds"))) return rc;
         }
     }
     const int rounds = g + 1;

@@ -147,7 +147,8 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
     // end) and give the other, cold slots a plain atomicMin
     const int kg = (PH == 2 && P.flatten) ? __ldg(&P.in->giant) : -1;
     long long gbest = kInf;
-    const bool guard_cold = PH == 2 ? (P.guards > 0 || (P.guards < 0 && ECL_P2_GUARD_COLD)) : guard;
+    // (no largest set: every slot may be hot -- guard them all, as in phase 1's guard rule)
+    const bool guard_cold = PH == 2 ? (P.guards > 0 || (P.guards < 0 && (ECL_P2_GUARD_COLD || kg < 0))) : guard;
     auto rec = [&](int x, long long key) {
         if (PH == 2 && x == kg) gbest = min(gbest, key);
         else record_min(D.k(x), key, guard_cold);

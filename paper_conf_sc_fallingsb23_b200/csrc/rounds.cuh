@@ -55,32 +55,33 @@ __global__ void __launch_bounds__(256) k_flatten(Params P) {
 }
 
 // After phase 1 most vertices of a graph whose light edges percolate (C3-C5)
-// sit in ONE set.  Find its root by a majority vote over sampled vertices.
+// sit in ONE set.  Find its root as the mode of 256 sampled vertices' roots.
 // The phase-2 populate keeps that set's key minimum per warp (it is the hot
 // slot almost every kept edge touches), and for n >= 2^25 k_flatten<2> writes
 // a bitmap of its members, so that populate filters an edge with both ends in
 // it from the bitmap (n/8 bytes, L2 resident) instead of two random parent
 // loads.
 __global__ void __launch_bounds__(256) k_giant(Params P) {
-    constexpr int kS = 256;   // samples (one per thread): a set holding >= 1/4 shows up reliably
+    constexpr int kS = 256;   // samples (one per thread)
     __shared__ int s_r[kS];
+    __shared__ int s_c[kS];
     if (!phase2_needed(P) || !P.flatten) return;
     const DS D = ds_of(P);
-    {
-        const int i = threadIdx.x;
-        const long long v = (long long)(splitmix64(0x6A09E667F3BCC909ull + (unsigned long long)i) % (unsigned long long)P.n);
-        s_r[i] = find_root(D, (int)v, false);
-    }
+    const int i = threadIdx.x;
+    const long long v = (long long)(splitmix64(0x6A09E667F3BCC909ull + (unsigned long long)i) % (unsigned long long)P.n);
+    s_r[i] = find_root(D, (int)v, false);
     __syncthreads();
-    if (threadIdx.x == 0) {
-        int cand = -1, votes = 0;                 // Boyer-Moore majority vote
-        for (int i = 0; i < kS; ++i) {
-            if (votes == 0) { cand = s_r[i]; votes = 1; }
-            else votes += (s_r[i] == cand) ? 1 : -1;
-        }
-        int cnt = 0;
-        for (int i = 0; i < kS; ++i) cnt += s_r[i] == cand;
-        P.in->giant = cnt >= kS / 4 ? cand : -1;   // worth it only if it holds >= 1/4
+    // the mode of the samples, exactly (a majority vote misses a set holding
+    // less than half of them, e.g. RMAT's giant among many isolated vertices)
+    int c = 0;
+    for (int t = 0; t < kS; ++t) c += s_r[t] == s_r[i];
+    s_c[i] = c;
+    __syncthreads();
+    if (i == 0) {
+        int best = 0;
+        for (int t = 1; t < kS; ++t)
+            if (s_c[t] > s_c[best] || (s_c[t] == s_c[best] && s_r[t] < s_r[best])) best = t;
+        P.in->giant = s_c[best] >= kS / 8 ? s_r[best] : -1;   // worth it only if it holds >= 1/8
     }
 }
 
