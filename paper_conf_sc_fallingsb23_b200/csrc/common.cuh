@@ -119,6 +119,20 @@ struct Params {
     int* tgt;                         // per vertex hook target (distributed rep pass)
     long long* const* keys_all;       // virtual shards: every shard's key array
     int nkeys;
+    int* hcnt;                        // per arena: deferred tuples of a crowded-round split (distributed path)
+    struct DistSplit* dsp;            // the split decision shared by all shards (distributed path)
+};
+
+// Crowded-round split on the distributed path (the sharded analogue of
+// k_rounds' split, SURVEY §8(e) + reading Q17).  Every decision is a
+// function of replicated or allreduced values, so all ranks agree.
+struct DistSplit {
+    long long cand[8];                // per quantile: min candidate over this rank's virtual shards (partial)
+    long long live_sum;               // live tuples over this rank's virtual shards (partial)
+    int T;                            // this round's split threshold (INT_MAX: no split)
+    int nested;                       // the split appends below tuples already deferred in its output buffer
+    int hb;                           // buffer holding deferred tuples (-1: none)
+    int pad;
 };
 
 __device__ __forceinline__ DS ds_of(const Params& P) {

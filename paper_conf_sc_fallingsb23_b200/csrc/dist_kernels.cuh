@@ -119,6 +119,13 @@ __global__ void __launch_bounds__(256) k_dist_reps2(Params P, const int* R, long
     }
 }
 
+// keep[x] = x is a root (the sets phase 2 can record keys at)
+__global__ void __launch_bounds__(256) k_dist_root_keep(Params P, unsigned char* keep) {
+    const long long stride = (long long)gridDim.x * blockDim.x;
+    for (long long x = (long long)blockIdx.x * blockDim.x + threadIdx.x; x < P.n; x += stride)
+        keep[x] = __ldcg(P.parent + x) == (int)x;
+}
+
 // order-preserving compaction R_next = [R[i] : keep[i]] over a fixed grid of
 // contiguous slices: counts per block, then each block offsets its slice by
 // the counts of the blocks before it (every rank computes the same list)
@@ -153,12 +160,20 @@ __global__ void __launch_bounds__(kCompactBlock) k_dist_count(long long nR, cons
 __global__ void __launch_bounds__(kCompactBlock) k_dist_compact(const int* R, long long nR, const unsigned char* keep,
                                                                 const int* bcnt, int* Rnext, long long* nnext,
                                                                 unsigned long long* reps,
-                                                                volatile long long* host_out) {
+                                                                volatile long long* host_out,
+                                                                const DistSplit* dsp) {
     __shared__ int s_base, s_w[kCompactBlock / 32];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    {   // this block's offset: the counts of the blocks before it (block-wide sum)
+        int b = 0;
+        for (unsigned k = threadIdx.x; k < blockIdx.x; k += kCompactBlock) b += bcnt[k];
+        b = warp_sum(b);
+        if (lane == 0) s_w[warp] = b;
+        __syncthreads();
+    }
     if (threadIdx.x == 0) {
         int b = 0;
-        for (unsigned k = 0; k < blockIdx.x; ++k) b += bcnt[k];
+        for (int w = 0; w < kCompactBlock / 32; ++w) b += s_w[w];
         s_base = b;
         if (blockIdx.x == gridDim.x - 1) {
             const long long nn = (long long)b + bcnt[blockIdx.x];
@@ -166,28 +181,122 @@ __global__ void __launch_bounds__(kCompactBlock) k_dist_compact(const int* R, lo
             if (host_out) {
                 host_out[0] = (long long)*reps;
                 host_out[1] = nn;
+                host_out[2] = dsp ? (long long)dsp->hb : -1;
             }
             *reps = 0;
         }
     }
     __syncthreads();
+    // each warp takes a contiguous piece of the block's slice: count it, then
+    // emit it in order after the pieces of the warps before it
     long long lo, hi;
     slice_of(nR, lo, hi);
-    for (long long i0 = lo; i0 < hi; i0 += kCompactBlock) {
-        const long long i = i0 + threadIdx.x;
-        const bool k = i < hi && keep[i];
+    constexpr int kW = kCompactBlock / 32;
+    const long long per = (hi - lo + kW - 1) / kW;
+    const long long wlo = min(hi, lo + warp * per), whi = min(hi, wlo + per);
+    int c = 0;
+    for (long long i = wlo + lane; i < whi; i += 32) c += keep[i];
+    c = warp_sum(c);
+    __shared__ int s_c[kW];
+    if (lane == 0) s_c[warp] = c;
+    __syncthreads();
+    int base = s_base;
+    for (int w = 0; w < warp; ++w) base += s_c[w];
+    const unsigned lt = (1u << lane) - 1u;
+    for (long long i0 = wlo; i0 < whi; i0 += 32) {
+        const long long i = i0 + lane;
+        const bool k = i < whi && keep[i];
         const unsigned m = __ballot_sync(kFull, k);
-        if (lane == 0) s_w[warp] = __popc(m);
-        __syncthreads();
-        int before = 0, tot = 0;
-        for (int w = 0; w < kCompactBlock / 32; ++w) {
-            before += w < warp ? s_w[w] : 0;
-            tot += s_w[w];
+        if (k) Rnext[base + __popc(m & lt)] = (int)set_of(R, i);
+        base += __popc(m);
+    }
+}
+
+// Split candidates of shard P (launched once per virtual shard, k = 0..S-1,
+// on live list `cur`, before that round's key exchange): from 512 samples
+// spread evenly over the shard's arenas (split_threshold's rule), the weight
+// of sample rank N / 2^j for j = 1..kSplitQ -- thresholds with about 2^-j of
+// the live tuples below them (INT_MAX if none lies below).  The last shard's
+// launch writes {-live tuples, candidates} behind the exchanged keys (ext),
+// so the key allreduce(min) also yields the largest rank's live count and
+// the smallest candidate of each quantile; k_dist_split_decide then picks
+// the quantile nearest c x winners / live once the round's winners are known.
+constexpr int kSplitQ = 8;
+constexpr int kSplitExt = 1 + kSplitQ;   // slots behind the exchanged keys
+__global__ void __launch_bounds__(512) k_dist_split_cand(Params P, int k, int S, int cur, long long* ext) {
+    constexpr int N = kSplitSamples;
+    __shared__ int s_w[N];
+    __shared__ long long s_live;
+    __shared__ int s_c[kSplitQ];
+    const int tid = threadIdx.x;
+    DistSplit* d = P.dsp;
+    const int4* base = cur ? P.wl1 : P.wl0;
+    if (tid == 0) s_live = 0;
+    if (tid < kSplitQ) s_c[tid] = INT_MAX;
+    __syncthreads();
+    {
+        long long l = 0;
+        for (int b = tid; b < P.G; b += blockDim.x) l += P.acnt[b];
+        l = warp_sum(l);
+        if ((tid & 31) == 0 && l) atomicAdd(reinterpret_cast<unsigned long long*>(&s_live), (unsigned long long)l);
+    }
+    __syncthreads();
+    const long long live = s_live;
+    if (live > 0) {
+        for (int i = tid; i < N; i += blockDim.x) {
+            const int b = (int)((long long)i * P.G / N);                // arena of sample i
+            const int i0 = (int)(((long long)b * N + P.G - 1) / P.G);   // its first sample
+            const int i1 = (int)(((long long)(b + 1) * N + P.G - 1) / P.G);
+            const int cnt = P.acnt[b], ks = i1 - i0, t = i - i0;
+            s_w[i] = cnt > 0 ? __ldcg(&base[(long long)b * P.cap + (long long)(2 * t + 1) * cnt / (2 * ks)].z) : INT_MAX;
         }
-        if (k) Rnext[s_base + before + __popc(m & ((1u << lane) - 1u))] = (int)set_of(R, i);
         __syncthreads();
-        if (threadIdx.x == 0) s_base += tot;
+        for (int i = tid; i < N; i += blockDim.x) {
+            const int wi = s_w[i];
+            int less = 0, rank = 0;
+            for (int t = 0; t < N; ++t) {
+                const int wt = s_w[t];
+                less += wt < wi;
+                rank += (wt < wi) || (wt == wi && t < i);
+            }
+            for (int j = 1; j <= kSplitQ; ++j)
+                if (rank == (N >> j)) s_c[j - 1] = (less > 0 && wi != INT_MAX) ? wi : INT_MAX;
+        }
         __syncthreads();
+    }
+    if (tid == 0) {
+        for (int j = 0; j < kSplitQ; ++j)
+            d->cand[j] = k == 0 ? (long long)s_c[j] : min(d->cand[j], (long long)s_c[j]);
+        d->live_sum = (k == 0 ? 0 : d->live_sum) + live;
+        if (k == S - 1) {
+            ext[0] = -d->live_sum;
+            for (int j = 0; j < kSplitQ; ++j) ext[1 + j] = d->cand[j];
+        }
+    }
+}
+
+// After the key allreduce and the rep passes of round g: pass A g + 1's
+// split threshold, the same on every rank.  The crowded rule is crowded()'s,
+// with the global live count estimated as ranks x the largest rank's count;
+// the threshold is the candidate quantile 2^-j closest to c x winners / live.
+__global__ void k_dist_split_decide(Params P, const long long* ext, int cur, int g, int world) {
+    if (threadIdx.x != 0) return;
+    DistSplit* d = P.dsp;
+    const long long live = -ext[0] * (long long)world;
+    const long long win = __ldcg(&P.st->winners[g]);
+    const int hb = d->hb;
+    int T = INT_MAX;
+    if ((hb < 0 || hb == (cur ^ 1)) && crowded(P, live, win, g + 1)) {
+        const double f = (double)ECL_SPLIT_C * (double)win / (double)max(live, 1LL);   // target light fraction
+        int j = 1;
+        while (j < kSplitQ && ldexp(1.0, -(j + 1)) >= f) ++j;                         // 2^-j >= f > 2^-(j+1)
+        if (f < 0.5) T = (int)min((long long)INT_MAX, ext[j]);
+    }
+    d->T = T;
+    d->nested = T != INT_MAX && hb >= 0;
+    if (T != INT_MAX) {
+        d->hb = cur ^ 1;
+        P.in->splits += 1;
     }
 }
 
@@ -207,12 +316,45 @@ __global__ void __launch_bounds__(kBlock, 2) k_dist_passA(Params P, int g, int c
         const RegionSrc R = region_src(P, b, s_pre, s_rcnt, s_red, &P.st->live[g - 1], g - 1 == 0);
         passA(P, R, wl[cur ^ 1], &s_out, P.guards != 0);
     } else {
+        // a crowded-round split (decided by k_dist_split_decide): light
+        // tuples to the front of the output arena, the rest deferred to its
+        // back (below the tuples deferred earlier when nested)
+        const int T = P.dsp ? __ldcg(&P.dsp->T) : INT_MAX;
+        __shared__ int s_def;
+        if (tid == 0) s_def = (T != INT_MAX && __ldcg(&P.dsp->nested)) ? P.hcnt[b] : 0;
         __syncthreads();
-        passA(P, compact_src(wl[cur], P.acnt[b]), wl[cur ^ 1], &s_out, P.guards != 0);
+        const CompactSrc S = compact_src(wl[cur], P.acnt[b]);
+        if (T != INT_MAX) {
+            passA<true>(P, S, wl[cur ^ 1], &s_out, P.guards != 0, T, wl[cur ^ 1] + P.cap, &s_def);
+            __syncthreads();
+            if (tid == 0) P.hcnt[b] = s_def;
+        } else {
+            passA(P, S, wl[cur ^ 1], &s_out, P.guards != 0);
+        }
     }
     __syncthreads();
     if (tid == 0) {
         P.acnt[b] = s_out;
+        if (s_out) atomicAdd(reinterpret_cast<unsigned long long*>(&P.st->live[g]), (unsigned long long)s_out);
+    }
+}
+
+// The light part of a split is done everywhere: filter this shard's deferred
+// tuples (back of buffer hb) into the front of buffer hb ^ 1 -- a pass A with
+// guards, since every key is inf again.
+__global__ void __launch_bounds__(kBlock, 2) k_dist_drain(Params P, int g, int hb) {
+    __shared__ int s_out;
+    const int tid = threadIdx.x;
+    const int b = blockIdx.x;
+    int4* wl[2] = {P.wl0 + (long long)b * P.cap, P.wl1 + (long long)b * P.cap};
+    if (tid == 0) s_out = 0;
+    __syncthreads();
+    const int h = P.hcnt[b];
+    passA(P, compact_src(wl[hb] + P.cap - h, h), wl[hb ^ 1], &s_out, true);
+    __syncthreads();
+    if (tid == 0) {
+        P.acnt[b] = s_out;
+        P.hcnt[b] = 0;
         if (s_out) atomicAdd(reinterpret_cast<unsigned long long*>(&P.st->live[g]), (unsigned long long)s_out);
     }
 }

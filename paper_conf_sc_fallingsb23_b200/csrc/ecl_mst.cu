@@ -275,6 +275,8 @@ static int run_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t
     P.zero_mst = 1;
     P.acnt = nullptr;
     P.tgt = nullptr;
+    P.hcnt = nullptr;
+    P.dsp = nullptr;
     P.keys_all = nullptr;
     P.nkeys = 1;
     if ((reinterpret_cast<uintptr_t>(nlist) | reinterpret_cast<uintptr_t>(eweight)) % 16 ||
@@ -597,7 +599,7 @@ struct DistHandle {
     int rank = 0, world = 1;
     NcclComm comm = nullptr;
     long long* h_pin = nullptr;   // pinned host words (phase-2 decision, stats)
-    long long* h_map = nullptr;   // mapped pinned pair {sets with a finite key, |R_next|}, written by k_dist_compact
+    long long* h_map = nullptr;   // mapped pinned {sets with a finite key, |R_next|, deferred buffer}, written by k_dist_compact
     long long* d_map = nullptr;   // its device alias
     cudaEvent_t ev = nullptr;     // recorded after k_dist_compact each round
 };
@@ -610,8 +612,8 @@ static void release(DistHandle* h) {
 }
 
 struct DistLayout {
-    size_t stats, internal, rowstart, parent, tgt, keyptrs, rl0, rl1, rbuf, keep, bcnt, shard0, shard_bytes, total;
-    size_t region, acnt, key, wl0, wl1;   // offsets inside one shard block
+    size_t stats, internal, rowstart, parent, tgt, keyptrs, rl0, rl1, rbuf, keep, bcnt, dsplit, giant, shard0, shard_bytes, total;
+    size_t region, acnt, hcnt, key, wl0, wl1;   // offsets inside one shard block
     long long wl_cap, nlocal_max;
 };
 
@@ -631,12 +633,15 @@ static inline DistLayout dist_layout(int64_t n, int64_t M, int S, int world) {
     L.keyptrs = off;  off = align_up(off + sizeof(long long*) * (size_t)S, 256);
     L.rl0 = off;      off = align_up(off + sizeof(int) * (size_t)n, 256);     // root lists (double buffer)
     L.rl1 = off;      off = align_up(off + sizeof(int) * (size_t)n, 256);
-    L.rbuf = off;     off = align_up(off + sizeof(long long) * (size_t)n, 256);   // the allreduce buffer
+    L.rbuf = off;     off = align_up(off + sizeof(long long) * ((size_t)n + kSplitExt), 256);   // the allreduce buffer (+ split extras)
     L.keep = off;     off = align_up(off + (size_t)n, 256);
     L.bcnt = off;     off = align_up(off + sizeof(int) * (size_t)kCompactGridMax, 256);
+    L.dsplit = off;   off = align_up(off + sizeof(DistSplit), 256);
+    L.giant = off;    off = align_up(off + sizeof(unsigned) * (size_t)((n + 31) / 32 + 1), 256);   // largest-set bitmap
     size_t so = 0;
     L.region = so; so = align_up(so + sizeof(int4) * (size_t)kMaxPopWarps, 256);
     L.acnt = so;   so = align_up(so + sizeof(int) * (size_t)kMaxGrid, 256);
+    L.hcnt = so;   so = align_up(so + sizeof(int) * (size_t)kMaxGrid, 256);
     L.key = so;    so = align_up(so + sizeof(long long) * (size_t)n, 256);
     L.wl0 = so;    so = align_up(so + sizeof(int4) * (size_t)L.wl_cap, 256);
     L.wl1 = so;    so = align_up(so + sizeof(int4) * (size_t)L.wl_cap, 256);
@@ -669,7 +674,7 @@ int ecl_mst_dist_init(const void* uid, int32_t rank, int32_t world, void** handl
     h->world = world;
     cudaError_t e = cudaHostAlloc(reinterpret_cast<void**>(&h->h_pin), sizeof(long long) * 4, cudaHostAllocDefault);
     if (e == cudaSuccess)
-        e = cudaHostAlloc(reinterpret_cast<void**>(&h->h_map), sizeof(long long) * 2, cudaHostAllocMapped);
+        e = cudaHostAlloc(reinterpret_cast<void**>(&h->h_map), sizeof(long long) * 4, cudaHostAllocMapped);
     if (e == cudaSuccess) e = cudaHostGetDevicePointer(reinterpret_cast<void**>(&h->d_map), h->h_map, 0);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->ev, cudaEventDisableTiming);
     if (e != cudaSuccess) {
@@ -757,6 +762,12 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
     const long long nchunks = ceil_div(M, kChunk);
     const long long Pt = (long long)S * world;
 
+    // crowded-round splits (opts.refilter, reading Q17): decided on the
+    // device from allreduced values, the same on every rank
+    // (auto: only where the two-phase filter is on too, M >= 4n -- the dense
+    // graphs whose giant set crowds the rounds; C2 x1 4.33 vs 3.80 ms with them)
+    const bool split_on = o.refilter > 0 || (o.refilter < 0 && (o.filter > 0 || (o.filter < 0 && M >= 4LL * n)));
+    DistSplit* dsp = reinterpret_cast<DistSplit*>(ws + L.dsplit);
     // per-shard launch geometry and parameters
     std::vector<Params> sp(S);
     std::vector<long long*> keyptr(S);
@@ -811,7 +822,7 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
         P.halving = o.path_halving ? 1 : 0;
         P.guards = o.atomic_guards == 0 ? 0 : 1;
         P.flatten = o.flatten ? 1 : 0;
-        P.refilter = 0;                 // the sharded rounds are host-driven (no split)
+        P.refilter = o.refilter < 0 ? -1 : (o.refilter ? 1 : 0);   // crowded-round split (Q17)
         P.samp = nullptr;
         P.shard = shard;
         P.nshards = (int)Pt;
@@ -819,6 +830,10 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
         P.zero_mst = 0;
         P.acnt = reinterpret_cast<int*>(sb + L.acnt);
         P.tgt = reinterpret_cast<int*>(ws + L.tgt);
+        P.hcnt = reinterpret_cast<int*>(sb + L.hcnt);
+        // phase 2: the largest set's bitmap where parent[] exceeds the L2, as on one GPU
+        P.giant_bits = (long long)n >= ECL_GIANT_MIN_N ? reinterpret_cast<unsigned*>(ws + L.giant) : nullptr;
+        P.dsp = split_on ? dsp : nullptr;
         P.keys_all = d_keyptrs;
         P.nkeys = S;
     }
@@ -845,11 +860,24 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
 
     if (e == cudaSuccess) e = cudaMemsetAsync(st, 0, sizeof(ecl_mst_stats), s);
     if (e == cudaSuccess) e = cudaMemsetAsync(in, 0, sizeof(Internal), s);   // (reps: zeroed again by each k_dist_compact)
+    if (e == cudaSuccess) e = cudaMemsetAsync(&dsp->hb, 0xFF, sizeof(int), s);    // hb = -1: nothing deferred
     if (e == cudaSuccess) e = cudaMemsetAsync(in_mst_out, 0, (size_t)M, s);   // every rank returns the full mask
     if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "memset: %s", cudaGetErrorString(e));
     k_init<<<vblocks, 256, 0, s>>>(P0);
     if ((rc = check("k_init"))) return rc;
     int g = 0;
+    int* const rlist[2] = {reinterpret_cast<int*>(ws + L.rl0), reinterpret_cast<int*>(ws + L.rl1)};
+    unsigned char* const rkeep = reinterpret_cast<unsigned char*>(ws + L.keep);
+    int* const rcnt = reinterpret_cast<int*>(ws + L.bcnt);
+    long long phase2_roots = 0;
+    // the current roots into `out` (count: h_map[1] after the next sync)
+    auto launch_roots = [&](int* out) {
+        const unsigned cb = (unsigned)std::max<long long>(1, std::min<long long>(ceil_div(n, 4096), kCompactGridMax));
+        k_dist_root_keep<<<vblocks, 256, 0, s>>>(P0, rkeep);
+        k_dist_count<<<cb, kCompactBlock, 0, s>>>(n, rkeep, rcnt);
+        k_dist_compact<<<cb, kCompactBlock, 0, s>>>(nullptr, n, rkeep, rcnt, out, &in->nroots, &in->reps, h->d_map,
+                                                    nullptr);
+    };
     for (int ph = 1; ph <= 2; ++ph) {
         if (ph == 2) {
             // the phase-2 decision needs the global deferred count
@@ -859,12 +887,18 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
             if ((rc = read_word(&st->filtered, &filtered))) return rc;
             if (!(filtered & 0xffffffffll) || heavy == 0) break;
             k_flatten<1><<<vblocks, 256, 0, s>>>(P0);
+            k_giant<<<1, 256, 0, s>>>(P0);   // replicated parent[]: every rank finds the same set
             k_flatten<2><<<vblocks, 256, 0, s>>>(P0);
+            // phase 2 records keys at roots only (set(u), set(v) after the
+            // flatten): its first exchange covers the roots, not all n
+            // vertices (C5: about 1 M of 67 M after phase 1)
+            launch_roots(rlist[0]);
             ++g;
             if (g >= ECL_MST_MAX_ROUNDS) return fail(ECL_MST_ERR_INPUT, "round limit");
             e = cudaMemcpyAsync(&st->phase2_round, &g, sizeof(int), cudaMemcpyHostToDevice, s);
             if (e == cudaSuccess) e = cudaStreamSynchronize(s);   // &g is a host stack value
             if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "phase2: %s", cudaGetErrorString(e));
+            phase2_roots = reinterpret_cast<volatile long long*>(h->h_map)[1];
         }
         for (int k = 0; k < S; ++k) {
             if (ph == 1) k_populate<1><<<(unsigned)ceil_div(sp[k].W, kPopWarps), kPopBlock, 0, s>>>(sp[k]);
@@ -875,13 +909,13 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
         int cur = 0;
         // the sets whose keys are exchanged: all n in the phase's first round,
         // then the roots that can still hold a live edge (root-compacted)
-        const int* R = nullptr;
-        long long nR = n;
-        int rb = 0;
-        int* rl[2] = {reinterpret_cast<int*>(ws + L.rl0), reinterpret_cast<int*>(ws + L.rl1)};
+        int* const* rl = rlist;
+        const int* R = ph == 2 ? rl[0] : nullptr;
+        long long nR = ph == 2 ? phase2_roots : n;
+        int rb = ph == 2 ? 1 : 0;
         long long* rbuf = reinterpret_cast<long long*>(ws + L.rbuf);
-        unsigned char* keep = reinterpret_cast<unsigned char*>(ws + L.keep);
-        int* bcnt = reinterpret_cast<int*>(ws + L.bcnt);
+        unsigned char* keep = rkeep;
+        int* bcnt = rcnt;
         // Each round is enqueued in full -- exchange, rep passes, root-list
         // compaction, and the next pass A -- before the host waits, on an
         // event behind the compaction, for the two words that decide the next
@@ -897,23 +931,31 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
             // A phase's first round exchanges all n keys: with one local shard
             // that is key[] itself, reduced in place (no gather/scatter copies;
             // reps2 resets key[x] only after reading it as buf[x]).
+            // With splits on, the split candidates of the live list ride
+            // behind the keys (kSplitExt slots; never in a phase's first round).
             long long* xbuf = rbuf;
-            if (R == nullptr && S == 1) {
+            const bool split = split_on && !first;
+            if (R == nullptr && S == 1 && !split) {
                 xbuf = P0.key;
                 if ((rc = allreduce(xbuf, (size_t)nR, kNcclMin))) return rc;
             } else {
+                if (split)
+                    for (int k = 0; k < S; ++k) k_dist_split_cand<<<1, 512, 0, s>>>(sp[k], k, S, cur, rbuf + nR);
                 k_dist_gather<<<rblocks, 256, 0, s>>>(P0, R, nR, rbuf);
-                if ((rc = allreduce(rbuf, (size_t)nR, kNcclMin))) return rc;
+                if ((rc = allreduce(rbuf, (size_t)nR + (split ? kSplitExt : 0), kNcclMin))) return rc;
                 k_dist_scatter<<<rblocks, 256, 0, s>>>(P0, R, nR, rbuf);
             }
             k_dist_reps1<<<rblocks, 256, 0, s>>>(P0, R, nR, xbuf);
             k_dist_reps2<<<rblocks, 256, 0, s>>>(P0, R, nR, xbuf, keep, g);
             k_dist_count<<<cblocks, kCompactBlock, 0, s>>>(nR, keep, bcnt);
-            k_dist_compact<<<cblocks, kCompactBlock, 0, s>>>(R, nR, keep, bcnt, rl[rb], &in->nroots, &in->reps, h->d_map);
+            k_dist_compact<<<cblocks, kCompactBlock, 0, s>>>(R, nR, keep, bcnt, rl[rb], &in->nroots, &in->reps, h->d_map,
+                                                             split_on ? dsp : nullptr);
             e = cudaEventRecord(h->ev, s);
             if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "event: %s", cudaGetErrorString(e));
             const bool can_continue = g + 1 < ECL_MST_MAX_ROUNDS;
             if (can_continue) {
+                if (split && !first)   // is pass A g + 1 a crowded round?  (from the allreduced extras)
+                    k_dist_split_decide<<<1, 32, 0, s>>>(P0, rbuf + nR, cur, g, world);
                 // (first: also counts the phase's populate output -- needed even
                 // when the phase turns out empty)
                 for (int k = 0; k < S; ++k) {
@@ -926,6 +968,27 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
             if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "sync: %s", cudaGetErrorString(e));
             const long long reps = reinterpret_cast<volatile long long*>(h->h_map)[0];
             const long long nnext = reinterpret_cast<volatile long long*>(h->h_map)[1];
+            const int hbv = (int)reinterpret_cast<volatile long long*>(h->h_map)[2];
+            if (reps == 0 && hbv >= 0) {
+                // the light part of a split is done on every rank: drain the
+                // deferred tuples (filter + record), then continue from the
+                // roots (their keys were inf in the empty round just ended)
+                if (g + 2 >= ECL_MST_MAX_ROUNDS) return fail(ECL_MST_ERR_INPUT, "round limit");
+                ++g;
+                for (int k = 0; k < S; ++k) k_dist_drain<<<sp[k].G, kBlock, 0, s>>>(sp[k], g, hbv);
+                e = cudaMemsetAsync(&dsp->hb, 0xFF, sizeof(int), s);
+                if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "memset: %s", cudaGetErrorString(e));
+                launch_roots(rl[0]);
+                e = cudaStreamSynchronize(s);
+                if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "sync: %s", cudaGetErrorString(e));
+                R = rl[0];
+                nR = reinterpret_cast<volatile long long*>(h->h_map)[1];
+                rb = 1;
+                cur = hbv ^ 1;
+                first = false;
+                if ((rc = check("drain"))) return rc;
+                continue;
+            }
             if (reps == 0) break;   // no set has a live edge anywhere: the phase is done
             if (!can_continue) return fail(ECL_MST_ERR_INPUT, "round limit");
             R = rl[rb];
@@ -937,7 +1000,8 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
         }
     }
     const int rounds = g + 1;
-    e = cudaMemcpyAsync(&st->rounds, &rounds, sizeof(int), cudaMemcpyHostToDevice, s);
+    e = cudaMemcpyAsync(&st->refilters, &in->splits, sizeof(int), cudaMemcpyDeviceToDevice, s);
+    if (e == cudaSuccess) e = cudaMemcpyAsync(&st->rounds, &rounds, sizeof(int), cudaMemcpyHostToDevice, s);
     if (e == cudaSuccess) e = cudaStreamSynchronize(s);
     if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "stats: %s", cudaGetErrorString(e));
     k_finalize<<<1, 32, 0, s>>>(P0);

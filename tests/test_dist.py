@@ -129,7 +129,7 @@ def test_sharded_matches_single_gpu_rounds(ecl):
     single = ecl.ecl_mst_read_stats(ws)
     h = ecl.ecl_mst_dist_init(None, 0, 1)
     try:
-        _, _, st = dist_run(ecl, g, h, 3)
+        _, _, st = dist_run(ecl, g, h, 3, refilter=0)
     finally:
         ecl.ecl_mst_dist_finalize(h)
     assert st["rounds"] == single["rounds"]
@@ -148,5 +148,42 @@ def test_one_rank_nccl_communicator(ecl):
             mask, total, st = dist_run(ecl, g, h, 1)
             omask, ototal, _ = oracle.kruskal_graph(g)
             assert total == ototal and np.array_equal(mask, omask)
+    finally:
+        ecl.ecl_mst_dist_finalize(h)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("shards", [1, 2, 5])
+@pytest.mark.parametrize("weights", ["ties", "two", "equal", "uniform"])
+def test_virtual_shards_refilter_forced(ecl, weights, shards):
+    """Crowded-round splits on the sharded path (opts.refilter = 1): the
+    threshold is agreed by an allreduce(min) over shards, light tuples run to
+    completion, deferred ones are drained and filtered -- same MSF."""
+    g = G.random_small(5000, 120000, seed=77 + shards, weights=weights, multi=True, self_loops=True)
+    omask, ototal, _ = oracle.kruskal_graph(g)
+    h = ecl.ecl_mst_dist_init(None, 0, 1)
+    try:
+        for opts in (dict(refilter=1), dict(refilter=1, filter=0), dict(refilter=1, filter_c=1)):
+            mask, total, st = dist_run(ecl, g, h, shards, **opts)
+            assert st["status"] == 0
+            assert total == ototal and np.array_equal(mask, omask), (shards, opts)
+            if weights == "uniform" and opts.get("filter") == 0:
+                assert st["refilters"] >= 1
+    finally:
+        ecl.ecl_mst_dist_finalize(h)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("name", ["rmat", "uniform"])
+def test_one_rank_nccl_refilter(ecl, name):
+    """Splits through a real NCCL communicator (the candidate allreduce)."""
+    uid = ecl.ecl_mst_dist_unique_id()
+    h = ecl.ecl_mst_dist_init(uid, 0, 1)
+    try:
+        g = synth.make_config(name, "small")
+        omask, ototal, _ = oracle.kruskal_graph(g)
+        for opts in (dict(refilter=1), dict(refilter=1, filter=0)):
+            mask, total, st = dist_run(ecl, g, h, 1, **opts)
+            assert total == ototal and np.array_equal(mask, omask), opts
     finally:
         ecl.ecl_mst_dist_finalize(h)
