@@ -30,13 +30,22 @@ sys.path.insert(0, ROOT)
 # directly, so fd 1 is pointed at stderr for the whole run and the JSON line
 # goes to a private duplicate of the original stdout.
 os.environ.setdefault("NCCL_DEBUG", "WARN")
-_JSON_OUT = os.fdopen(os.dup(1), "w")
-os.dup2(2, 1)
+_JSON_OUT = None
+
+
+def claim_stdout():
+    """Point fd 1 at stderr; keep a private handle on the original stdout."""
+    global _JSON_OUT
+    if _JSON_OUT is None:
+        _JSON_OUT = os.fdopen(os.dup(1), "w")
+        sys.stdout.flush()
+        os.dup2(2, 1)
 
 
 def emit(line):
-    _JSON_OUT.write(json.dumps(line) + "\n")
-    _JSON_OUT.flush()
+    out = _JSON_OUT if _JSON_OUT is not None else sys.stdout
+    out.write(json.dumps(line) + "\n")
+    out.flush()
 
 
 import torch  # noqa: E402
@@ -507,4 +516,5 @@ def main():
 
 
 if __name__ == "__main__":
+    claim_stdout()
     main()
