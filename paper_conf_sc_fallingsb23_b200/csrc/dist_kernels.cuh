@@ -60,17 +60,16 @@ __global__ void __launch_bounds__(256) k_dist_scatter(Params P, const int* R, lo
         P.key[set_of(R, i)] = buf[i];
 }
 
-// rep pass 1: for every set x = R[i] with a finite (reduced) key, the other
-// end's set q of its lightest edge, and whether that edge is q's lightest too
-// (mutual)
-__global__ void __launch_bounds__(256) k_dist_reps1(Params P, const int* R, long long nR, const long long* buf) {
+// rep pass 1: for every set x = R[i], i in [lo, hi), with a finite (reduced)
+// key, the other end's set q of its lightest edge, and whether that edge is
+// q's lightest too (mutual).  Ranks split R into slices and allgather tgt[].
+__global__ void __launch_bounds__(256) k_dist_reps1(Params P, const int* R, long long lo, long long hi,
+                                                    const long long* buf) {
     const long long stride = (long long)gridDim.x * blockDim.x;
-    unsigned long long found = 0;
-    for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < nR; i += stride) {
+    for (long long i = lo + (long long)blockIdx.x * blockDim.x + threadIdx.x; i < hi; i += stride) {
         const long long kx = buf[i];
         if (kx == kInf) continue;
         const long long x = set_of(R, i);
-        ++found;
         const unsigned j = (unsigned)(kx & 0xffffffffll);
         const int u = row_of_entry(P, (long long)j);
         const int v = __ldg(P.nlist + j);
@@ -80,8 +79,6 @@ __global__ void __launch_bounds__(256) k_dist_reps1(Params P, const int* R, long
         const bool mutual = P.key[q] == kx;
         P.tgt[i] = q | (mutual ? (int)0x80000000 : 0);
     }
-    found = warp_sum(found);
-    if ((threadIdx.x & 31) == 0 && found) atomicAdd(reinterpret_cast<unsigned long long*>(&P.in->reps), found);
 }
 
 // rep pass 2 (L30-31, L34-37): hook, mark, sum, reset -- the same rule as the
@@ -91,6 +88,7 @@ __global__ void __launch_bounds__(256) k_dist_reps2(Params P, const int* R, long
                                                     unsigned char* keep, int g) {
     const long long stride = (long long)gridDim.x * blockDim.x;
     long long wsum = 0, wcnt = 0;
+    unsigned long long found = 0;   // sets with a finite key (0: the phase is done)
     for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < nR; i += stride) {
         const long long kx = buf[i];
         const long long x = set_of(R, i);
@@ -98,6 +96,7 @@ __global__ void __launch_bounds__(256) k_dist_reps2(Params P, const int* R, long
             keep[i] = 0;
             continue;
         }
+        ++found;
         const int t = P.tgt[i];
         const int q = t & 0x7fffffff;
         const bool mutual = t < 0;
@@ -112,6 +111,8 @@ __global__ void __launch_bounds__(256) k_dist_reps2(Params P, const int* R, long
     }
     wsum = warp_sum(wsum);
     wcnt = warp_sum(wcnt);
+    found = warp_sum(found);
+    if ((threadIdx.x & 31) == 0 && found) atomicAdd(reinterpret_cast<unsigned long long*>(&P.in->reps), found);
     if ((threadIdx.x & 31) == 0 && wcnt) {
         atomicAdd(reinterpret_cast<unsigned long long*>(&P.st->total_weight), (unsigned long long)wsum);
         atomicAdd(reinterpret_cast<unsigned long long*>(&P.st->msf_edges), (unsigned long long)wcnt);

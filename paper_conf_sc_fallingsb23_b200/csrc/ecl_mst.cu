@@ -568,10 +568,11 @@ struct NcclApi {
     int (*getUniqueId)(NcclUid*) = nullptr;
     int (*commInitRank)(NcclComm*, int, NcclUid, int) = nullptr;
     int (*allReduce)(const void*, void*, size_t, int, int, NcclComm, cudaStream_t) = nullptr;
+    int (*allGather)(const void*, void*, size_t, int, NcclComm, cudaStream_t) = nullptr;
     int (*commDestroy)(NcclComm) = nullptr;
     const char* (*getErrorString)(int) = nullptr;
 };
-constexpr int kNcclInt64 = 4, kNcclSum = 0, kNcclMin = 3;
+constexpr int kNcclInt32 = 2, kNcclInt64 = 4, kNcclSum = 0, kNcclMin = 3;
 static NcclApi g_nccl;
 static std::mutex g_nccl_mu;
 
@@ -587,9 +588,11 @@ static int load_nccl() {
     g_nccl.commInitRank = reinterpret_cast<int (*)(NcclComm*, int, NcclUid, int)>(dlsym(h, "ncclCommInitRank"));
     g_nccl.allReduce = reinterpret_cast<int (*)(const void*, void*, size_t, int, int, NcclComm, cudaStream_t)>(
         dlsym(h, "ncclAllReduce"));
+    g_nccl.allGather = reinterpret_cast<int (*)(const void*, void*, size_t, int, NcclComm, cudaStream_t)>(
+        dlsym(h, "ncclAllGather"));
     g_nccl.commDestroy = reinterpret_cast<int (*)(NcclComm)>(dlsym(h, "ncclCommDestroy"));
     g_nccl.getErrorString = reinterpret_cast<const char* (*)(int)>(dlsym(h, "ncclGetErrorString"));
-    if (!g_nccl.getUniqueId || !g_nccl.commInitRank || !g_nccl.allReduce || !g_nccl.commDestroy)
+    if (!g_nccl.getUniqueId || !g_nccl.commInitRank || !g_nccl.allReduce || !g_nccl.allGather || !g_nccl.commDestroy)
         return fail(ECL_MST_ERR_CUDA, "libnccl.so.2 lacks the needed symbols");
     g_nccl.ok = true;
     return ECL_MST_OK;
@@ -629,7 +632,7 @@ static inline DistLayout dist_layout(int64_t n, int64_t M, int S, int world) {
     L.internal = off; off = align_up(off + sizeof(Internal), 256);
     L.rowstart = off; off = align_up(off + sizeof(int) * (size_t)(nchunks + 1), 256);
     L.parent = off;   off = align_up(off + sizeof(int) * (size_t)n, 256);
-    L.tgt = off;      off = align_up(off + sizeof(int) * (size_t)n, 256);
+    L.tgt = off;      off = align_up(off + sizeof(int) * ((size_t)n + world), 256);   // (+ allgather padding)
     L.keyptrs = off;  off = align_up(off + sizeof(long long*) * (size_t)S, 256);
     L.rl0 = off;      off = align_up(off + sizeof(int) * (size_t)n, 256);     // root lists (double buffer)
     L.rl1 = off;      off = align_up(off + sizeof(int) * (size_t)n, 256);
@@ -945,7 +948,21 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
                 if ((rc = allreduce(rbuf, (size_t)nR + (split ? kSplitExt : 0), kNcclMin))) return rc;
                 k_dist_scatter<<<rblocks, 256, 0, s>>>(P0, R, nR, rbuf);
             }
-            k_dist_reps1<<<rblocks, 256, 0, s>>>(P0, R, nR, xbuf);
+            // rep pass 1 -- the row search and finds, the costly part -- is
+            // split over the ranks (and over the virtual shards, which share
+            // tgt[]), then tgt[] is allgathered; pass 2 is replicated
+            if (nR > 0) {
+                const long long parts = world > 1 ? world : S;
+                const long long slice = ceil_div(nR, parts);
+                const unsigned sblocks = (unsigned)std::max<long long>(1, std::min<long long>(ceil_div(slice, 256), (long long)di.sms * 8));
+                for (long long k = (world > 1 ? rank : 0); k < (world > 1 ? rank + 1 : parts); ++k)
+                    k_dist_reps1<<<sblocks, 256, 0, s>>>(P0, R, std::min(nR, k * slice), std::min(nR, (k + 1) * slice), xbuf);
+                if (world > 1 && h->comm) {
+                    int* tg = P0.tgt;
+                    const int r = g_nccl.allGather(tg + (size_t)rank * slice, tg, (size_t)slice, kNcclInt32, h->comm, s);
+                    if (r) return fail(ECL_MST_ERR_CUDA, "ncclAllGather: %s", g_nccl.getErrorString ? g_nccl.getErrorString(r) : "?");
+                }
+            }
             k_dist_reps2<<<rblocks, 256, 0, s>>>(P0, R, nR, xbuf, keep, g);
             k_dist_count<<<cblocks, kCompactBlock, 0, s>>>(nR, keep, bcnt);
             k_dist_compact<<<cblocks, kCompactBlock, 0, s>>>(R, nR, keep, bcnt, rl[rb], &in->nroots, &in->reps, h->d_map,
