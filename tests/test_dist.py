@@ -187,3 +187,26 @@ def test_one_rank_nccl_refilter(ecl, name):
             assert total == ototal and np.array_equal(mask, omask), opts
     finally:
         ecl.ecl_mst_dist_finalize(h)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("seed", range(16))
+def test_virtual_shards_fuzz(ecl, seed):
+    """Random multigraphs with loops and tie-heavy weights through every
+    sharded-path mechanism at once: 2-4 virtual shards (rep pass 1 sliced
+    over them), forced crowded-round splits with drains, both phases."""
+    kinds = ["ties", "two", "equal", "full", "uniform"]
+    n = 50 + 97 * seed
+    g = G.random_small(n, 6 * n + 11 * seed, seed=900 + seed, weights=kinds[seed % 5], multi=True,
+                       self_loops=seed % 2 == 0)
+    omask, ototal, ocount = oracle.kruskal_graph(g)
+    h = ecl.ecl_mst_dist_init(None, 0, 1)
+    try:
+        for opts in (dict(refilter=1), dict(refilter=1, filter=1, threshold_mode=1, threshold=0),
+                     dict(refilter=1, filter=0, filter_c=1), dict(refilter=0)):
+            mask, total, st = dist_run(ecl, g, h, 2 + seed % 3, **opts)
+            assert st["status"] == 0, opts
+            assert total == ototal and np.array_equal(mask, omask), opts
+            assert st["msf_edges"] == ocount, opts
+    finally:
+        ecl.ecl_mst_dist_finalize(h)
