@@ -203,6 +203,49 @@ def test_host_api_staged_upload(eclmst, name):
         assert np.array_equal(out.numpy(), omask)
 
 
+def _star(leaves, seed=3):
+    # vertex 0 joined to every leaf: row 0 has `leaves` entries
+    n = leaves + 1
+    g = torch.Generator().manual_seed(seed)
+    w = torch.randint(0, 1000, (leaves,), generator=g, dtype=torch.int32)   # ties on purpose
+    nindex = torch.empty(n + 1, dtype=torch.int64)
+    nindex[0] = 0
+    nindex[1] = leaves
+    nindex[2:] = leaves + torch.arange(1, n, dtype=torch.int64)
+    nlist = torch.cat([torch.arange(1, n, dtype=torch.int32), torch.zeros(leaves, dtype=torch.int32)])
+    eweight = torch.cat([w, w])
+    return n, nindex, nlist, eweight
+
+
+@pytest.mark.parametrize("leaves", [300, 70000])   # a hub row below and above 2^16 entries
+def test_host_api_hub_rows(eclmst, leaves):
+    """A star (one row holding every edge) through the host path, pinned and
+    pageable: the staged upload's pieces split inside the hub row."""
+    n, nindex, nlist, eweight = _star(leaves)
+    omask, ototal, ocount = oracle.kruskal(n, nindex.numpy(), nlist.numpy(), eweight.numpy())
+    assert ocount == leaves
+    for pin in (True, False):
+        args = (nindex, nlist, eweight)
+        out = torch.empty(nlist.numel(), dtype=torch.uint8)
+        if pin:
+            args = tuple(a.pin_memory() for a in args)
+            out = out.pin_memory()
+        total = eclmst.ecl_mst(n, *args, out)
+        assert total == ototal
+        assert np.array_equal(out.numpy(), omask)
+
+
+def test_host_api_non_monotone_offsets(eclmst):
+    """Decreasing row offsets through the host path: the device validation
+    reports the inconsistent CSR."""
+    g = synth.make_config("grid", "small")
+    bad = g.nindex.clone()
+    bad[10], bad[11] = bad[11].item(), bad[10].item()
+    out = torch.empty(g.M, dtype=torch.uint8)
+    with pytest.raises(eclmst.EclMstError):
+        eclmst.ecl_mst(g.n, bad, g.nlist, g.eweight, out)
+
+
 def test_host_api_memcpy_variant(eclmst):
     g = synth.make_config("road", "small")
     omask, ototal, _ = oracle.kruskal_graph(g)
