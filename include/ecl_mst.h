@@ -84,9 +84,10 @@ typedef struct ecl_mst_options {
                                 tuples and > 6 per MSF edge of the last round; 0 never; 1 whenever
                                 live > 4 x last round's MSF edges (tests).  Same MSF either way. */
     int32_t filter_c;        /* c of P:143: the threshold targets the c|V| lightest CSR entries.
-                                0 (default) = 4, "we use c = 4 in our code"; P:394 aims
-                                for 3; "values between 2 and 4 seem to work well".  Only
-                                speed depends on it. */
+                                0 (default) auto: 3 when M >= 16n (P:394 and P:408 aim for "3
+                                times"), else 4 ("we use c = 4 in our code"); "values
+                                between 2 and 4 seem to work well".  Only speed depends
+                                on it. */
 } ecl_mst_options;
 
 /* per-run statistics written by the device into the workspace */

@@ -158,6 +158,14 @@ static int run_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t
                       uint8_t* in_mst_out, int64_t* total_weight_out, void* workspace, size_t workspace_bytes,
                       const ecl_mst_options* opts, void* stream, const Staging* stg);
 
+// c of P:143 (reading Q5b): opts.filter_c if set; else the paper's target of
+// "3 times" on dense graphs (M >= 16 n: C4/C5, where the light
+// part then still holds most MSF edges) and its code's c = 4 below.
+static inline int filter_c_for(int32_t opt, int32_t n, int64_t M) {
+    if (opt > 0) return opt;
+    return M >= 16LL * n ? 3 : 4;
+}
+
 extern "C" {
 
 int ecl_mst_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t* nlist, const int32_t* eweight,
@@ -263,7 +271,7 @@ static int run_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t
     P.threshold_mode = o.threshold_mode;
     P.threshold_value = o.threshold;
     P.samples = o.threshold_samples > 0 ? std::min(o.threshold_samples, kMaxSamples) : 20;
-    P.filter_c = o.filter_c > 0 ? o.filter_c : 4;
+    P.filter_c = filter_c_for(o.filter_c, n, M);
     P.halving = o.path_halving ? 1 : 0;
     P.guards = o.atomic_guards < 0 ? -1 : (o.atomic_guards ? 1 : 0);
     P.flatten = o.flatten ? 1 : 0;
@@ -821,7 +829,7 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
         P.threshold_mode = o.threshold_mode;
         P.threshold_value = o.threshold;
         P.samples = o.threshold_samples > 0 ? std::min(o.threshold_samples, kMaxSamples) : 20;
-        P.filter_c = o.filter_c > 0 ? o.filter_c : 4;
+        P.filter_c = filter_c_for(o.filter_c, n, M);
         P.halving = o.path_halving ? 1 : 0;
         P.guards = o.atomic_guards == 0 ? 0 : 1;
         P.flatten = o.flatten ? 1 : 0;
