@@ -495,6 +495,8 @@ def main():
                      "frac": achieved / peak, "traffic": traffic, "peak_source": peak_src,
                      "kernel": KERNEL_OF_STAGE.get(dominant, "all (sharded step)"), "stage": dominant,
                      "kernel_share_of_step": kern_ms.get(dominant, ms_max) / ms,
+                     # DRAM bytes of that kernel (ncu, committed summary) over its live event time
+                     "dram_frac": (traffic / (kern_ms.get(dominant, ms_max) / 1e3) / 1e9 / peak) if traffic else None,
                      "algorithmic_bytes_per_launch": ab[dominant],
                      "whole_step": {"algorithmic_bytes": ab["total"],
                                     "achieved_gbs": ab["total"] / (ms / 1e3) / 1e9,
