@@ -340,7 +340,8 @@ __device__ __forceinline__ bool use_guard(const Params& P, long long live, long 
 #define ECL_CROWD_RATIO 6    // auto: split when live > this x last round's MSF edges (C5: 56.8 -> 54.6 ms vs 16)
 #endif
 #ifndef ECL_SPLIT_C
-#define ECL_SPLIT_C 4        // light part: about this many edges per MSF edge of the last round
+#define ECL_SPLIT_C 2        // light part: about this many edges per MSF edge of the last round
+                             // (4 -> 2: C4 7.18 -> 7.10 ms, C2 2.283 -> 2.262 ms, C5 -0.5%, C3 +-0)
 #endif
 __device__ __forceinline__ bool crowded(const Params& P, long long live, long long winners, int g) {
     if (P.refilter == 0 || __ldcg(&P.in->splits) >= 16 || g + 24 >= ECL_MST_MAX_ROUNDS) return false;
@@ -348,8 +349,8 @@ __device__ __forceinline__ bool crowded(const Params& P, long long live, long lo
     return live >= (1LL << 20) && live > ECL_CROWD_RATIO * winners;
 }
 
-// T' such that about c = 4 live edges per set (4 x last round's MSF edges,
-// the paper's c = 4 of P:143 applied to the contracted graph) have w < T':
+// T' such that about c = ECL_SPLIT_C live edges per set (c x last round's MSF edges,
+// P:143's c applied to the contracted graph; 2, the low end of its range) have w < T':
 // every CTA samples its own worklist evenly, then every CTA ranks the same
 // samples (identical result everywhere).  INT_MAX: no useful split.  All
 // threads of all CTAs must call it (one grid barrier).
