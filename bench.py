@@ -6,8 +6,12 @@ MSF computation (all hot-path stages: init, threshold, populate, rounds,
 phase 2) over the workload graph, resident in HBM.  Edges/s counts CSR
 entries per second, the paper's throughput convention (Table 2).
 
-Workload at N=1: BASELINE configs[1], the road-network-like graph (C2,
-24M vertices, ~57.6M CSR entries); --config selects another family.
+Workload at N=1: BASELINE configs[4], the uniform random graph (C5, 2^26
+vertices, 2.0e9 CSR entries) -- the config the metric "at 1/2/4/8 B200" is
+quoted on; it fits one B200.  --config selects another family.  The whole
+graph is checked against the CPU oracle (serial Kruskal) in the same run, and
+that run's time is the cpu_baseline (about 4-5 minutes for C5; --parity none
+times a bounded sample instead).
 
   python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
 """
@@ -51,10 +55,18 @@ def emit(line):
 import torch  # noqa: E402
 
 PEAKS_FILE = os.path.join(ROOT, "MEASURED_PEAKS.json")
-# k_init, k_populate<1>, k_rounds<1>, k_finalize; with filtering also k_flatten<1>, k_flatten<2>,
-# k_populate<2>, k_rounds<2>
-LAUNCHES_UNFILTERED, LAUNCHES_FILTERED = 4, 8
+# k_init, k_populate<1>, k_rounds<1>, k_finalize; with filtering also k_flatten<1>, k_giant,
+# k_flatten<2>, k_populate<2>, k_rounds<2>
+LAUNCHES_UNFILTERED, LAUNCHES_FILTERED = 4, 9
 CONFIG_NAMES = {"grid": "C1", "road": "C2", "rgg": "C3", "rmat": "C4", "uniform": "C5"}
+# (graph name, n, M, m) of the full-size configs: pure functions of their seeds
+# (synth/); the GPU arm checks them against the generated graph, the
+# reference arm uses them to describe the same workload without building it
+FULL_SIZES = {"grid": ("grid512x512", 262144, 1046528, 523264),
+              "road": ("road6000x4000", 24000000, 57589978, 28794989),
+              "rgg": ("rgg16777216", 16777216, 100621104, 50310552),
+              "rmat": ("rmat24", 16777216, 520764976, 260382488),
+              "uniform": ("uniform67108864", 67108864, 1999999536, 999999768)}
 METRIC = "MSF edges/sec and ms/graph"
 KERNEL_OF_STAGE = {"init": "k_init", "populate1": "k_populate<1>", "rounds1": "k_rounds<1>",
                    "flatten": "k_flatten<1,2>", "populate2": "k_populate<2>", "rounds2": "k_rounds<2>",
@@ -67,11 +79,13 @@ def parse():
     ap.add_argument("--steps", type=int, default=9)     # the paper reports the median of 9 runs
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--config", default="road", choices=list(CONFIG_NAMES))
+    ap.add_argument("--config", default="uniform", choices=list(CONFIG_NAMES))
     ap.add_argument("--size", default="full", choices=["full", "small"])
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-parity", action="store_true")
+    ap.add_argument("--parity", default="full", choices=["full", "none"],
+                    help="full: the oracle on the whole benchmarked graph (mask + total), timed as cpu_baseline")
     ap.add_argument("--flush-mb", type=int, default=512)
     ap.add_argument("--opt", action="append", default=[], help="ecl_mst_options field=value (ablations)")
     ap.add_argument("--dist", action="store_true", help="use the edge-sharded NCCL path even on one GPU")
@@ -213,14 +227,33 @@ def stage_times(st: dict) -> dict:
     return out
 
 
-ORACLE_FULL_MAX_M = 120_000_000
+SAMPLE_MAX_M = 120_000_000
 
 
 def cpu_sample_graph(config):
+    """A bounded sample of the workload for the CPU oracle (about 5-10 s of
+    serial Kruskal): the same generator and density at a smaller size."""
     import synth
     kw = {"grid": dict(), "road": dict(), "rgg": dict(n=1 << 22),
-          "rmat": dict(scale=21, edge_factor=16), "uniform": dict(n=1 << 22, m_draws=30_000_000)}[config]
+          "rmat": dict(scale=21, edge_factor=16), "uniform": dict(n=1 << 21, m_draws=15 << 21)}[config]
     return synth.make_config(config, "full", **kw)
+
+
+def workload_config(args, world, use_dist, opt_kw, name, n, M, m):
+    """The `config` object of the JSON line; both arms print the same one."""
+    return {"workload": f"{CONFIG_NAMES[args.config]} {name}", "n": n, "M": M, "m_undirected": m,
+            "parallelism": (f"edge-sharded x{world} (ncclAllReduce min per round, replicated union-find)"
+                            if use_dist else "single GPU"),
+            "options": opt_kw,
+            "l2": (f"inputs ({(8 * M + 8 * n) / 1e6:.0f} MB CSR) "
+                   f"{'exceed' if 8 * M + 8 * n > 126e6 else 'fit in'} the 126 MB L2; a {args.flush_mb} MB "
+                   "buffer is written between steps (L2 flush)")}
+
+
+def full_size(args):
+    if args.size == "full":
+        return FULL_SIZES[args.config]
+    return None
 
 
 def load_peaks():
@@ -254,7 +287,19 @@ def run_reference(args, rank, world):
     import numpy as np  # noqa: F401
     import oracle
     import synth
-    g = synth.make_config(args.config, args.size)
+    fs = full_size(args)
+    if fs is not None and fs[2] > SAMPLE_MAX_M:
+        # one serial oracle run of the whole graph takes minutes (C5: ~5):
+        # each step is a bounded sample of the workload instead
+        g = cpu_sample_graph(args.config)
+        name, n_full, M_full, m_full = fs
+        sample = (f"{g.name} ({g.M} CSR entries), a smaller instance of the same generator and density, "
+                  f"per step; serial C Kruskal (oracle/kruskal.c)")
+    else:
+        g = synth.make_config(args.config, args.size)
+        name, n_full, M_full = g.name, g.n, g.M
+        m_full = fs[3] if fs else None
+        sample = f"whole {g.name} graph per step (serial C Kruskal, oracle/kruskal.c)"
     n, nindex, nlist, eweight = g.numpy()
     times = []
     for i in range(args.warmup + args.steps):
@@ -265,13 +310,14 @@ def run_reference(args, rank, world):
             times.append(dt)
     ms = 1e3 * sum(times) / len(times)
     value = g.M / (ms / 1e3)
+    opt_kw = {k: int(v) for k, v in (o.split("=", 1) for o in args.opt)}
+    use_dist = world > 1 or args.dist
     line = {
         "impl": "reference", "metric": METRIC, "value": value, "unit": "edges/s", "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
-        "config": {"workload": f"{CONFIG_NAMES[args.config]} {g.name}", "n": g.n, "M": g.M},
-        "cpu_baseline": {"value": value, "unit": "edges/s", "cores": 1, "kind": "oracle",
-                         "sample": f"whole {g.name} graph per step (serial C Kruskal, oracle/kruskal.c)"},
+        "config": workload_config(args, world, use_dist, opt_kw, name, n_full, M_full, m_full),
+        "cpu_baseline": {"value": value, "unit": "edges/s", "cores": 1, "kind": "oracle", "sample": sample},
         "e2e": {"value": value, "unit": "edges/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     emit(line)
@@ -306,6 +352,10 @@ def main():
     torch.cuda.synchronize()
     t_gen = time.perf_counter() - t_gen
     n, M = g.n, g.M
+    gname = g.name
+    fs = full_size(args)
+    if fs is not None and (fs[0], fs[1], fs[2]) != (g.name, n, M):
+        raise RuntimeError(f"generator drift: {(g.name, n, M)} != FULL_SIZES {fs[:3]}")
 
     handle = None
     if use_dist:   # edge-sharded path: NCCL allreduce(min) per round inside the library
@@ -371,6 +421,7 @@ def main():
     # ---- e2e through the host C-ABI call (pinned host buffers, copies timed) ----
     e2e = None
     in_mst_h = None
+    h_csr = None
     if not args.no_e2e and use_dist:
         # sharded e2e through the public API: pinned host CSR -> device, run, mask -> host
         h_idx = g.nindex.cpu().pin_memory()
@@ -422,7 +473,9 @@ def main():
         e_ms = 1e3 * sum(et) / len(et)
         e2e = {"value": M / (e_ms / 1e3), "unit": "edges/s",
                "h2d_bytes_per_step": 8 * (n + 1) + 8 * M, "d2h_bytes_per_step": M + 8,
-               "ms_per_step": e_ms, "same_result": tot_h == result_total}
+               "ms_per_step": e_ms, "same_result": tot_h == result_total and torch.equal(h_out, in_mst_h),
+               "path": "ecl_mst (host C-ABI call, P:325 memcpy variant) on pinned host buffers"}
+        h_csr = (h_idx, h_list, h_w)   # the oracle reads the same host arrays
 
     if rank != 0:
         if use_dist:
@@ -431,28 +484,36 @@ def main():
         return
 
     # ---- parity + cpu baseline: the oracle on the same arrays (rank 0, N=1 only) ----
+    # --parity full: one serial Kruskal over the whole benchmarked graph, after
+    # the GPU legs (nothing else runs meanwhile); it is both the parity check
+    # (mask + total) and the cpu_baseline (same workload, 1 core).
     parity = None
     cpu_baseline = None
-    if world == 1 and not (args.no_cpu_baseline and args.no_parity):
+    want_parity = args.parity == "full" and not args.no_parity
+    if world == 1 and (want_parity or not args.no_cpu_baseline):
         import numpy as np
         import oracle
-        if M <= ORACLE_FULL_MAX_M:
-            hn, hidx, hlist, hw = g.numpy()
+        if want_parity:
+            if h_csr is not None:
+                hn, hidx, hlist, hw = n, h_csr[0].numpy(), h_csr[1].numpy(), h_csr[2].numpy()
+            else:
+                hn, hidx, hlist, hw = g.numpy()
             t0 = time.perf_counter()
-            omask, ototal, _ = oracle.kruskal(hn, hidx, hlist, hw)
+            omask, ototal, ocount = oracle.kruskal(hn, hidx, hlist, hw)
             o_s = time.perf_counter() - t0
-            if not args.no_parity:
-                parity = bool(ototal == result_total and np.array_equal(omask, (in_mst_h if in_mst_h is not None else in_mst.cpu()).numpy()))
-            sample_desc = f"whole {g.name} graph, one serial C Kruskal run (oracle/kruskal.c)"
+            gmask = (in_mst_h if in_mst_h is not None else in_mst.cpu()).numpy()
+            parity = bool(ototal == result_total and ocount == st["msf_edges"] and np.array_equal(omask, gmask))
+            del omask, gmask
+            sample_desc = f"the whole benchmarked graph ({gname}), one serial C Kruskal run (oracle/kruskal.c)"
             sample_M = M
         else:
-            # bounded sample: the same family at a size the serial oracle finishes in ~10-30 s
-            gs = cpu_sample_graph(args.config)
+            # bounded sample: the same family at a size the serial oracle finishes in ~5-10 s
+            gs = cpu_sample_graph(args.config) if M > SAMPLE_MAX_M else synth.make_config(args.config, args.size)
             hn, hidx, hlist, hw = gs.numpy()
             t0 = time.perf_counter()
             oracle.kruskal(hn, hidx, hlist, hw)
             o_s = time.perf_counter() - t0
-            sample_desc = (f"{gs.name} ({gs.M} CSR entries), a smaller instance of the same generator, "
+            sample_desc = (f"{gs.name} ({gs.M} CSR entries), an instance of the same generator, "
                            f"one serial C Kruskal run (oracle/kruskal.c); full-size parity is in tests/")
             sample_M = gs.M
         if not args.no_cpu_baseline:
@@ -470,7 +531,7 @@ def main():
         ab["total_step"] = ab["total"]
         dominant = "total_step"
     achieved = ab[dominant] / (kern_ms.get(dominant, ms_max) / 1e3) / 1e9
-    prof = load_traffic(g.name)
+    prof = load_traffic(gname)
     traffic = None
     if prof:
         traffic = prof.get("dram_bytes_per_launch", {}).get(dominant)
@@ -479,16 +540,10 @@ def main():
         "metric": METRIC, "value": value, "unit": "edges/s", "n_gpus": world, "steps": args.steps,
         "warmup": max(args.warmup, 3), "ms_per_step": ms_max, "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
-        "config": {"workload": f"{CONFIG_NAMES[args.config]} {g.name}", "n": n, "M": M,
-                   "m_undirected": st["canonical_edges"],
-                   "parallelism": (f"edge-sharded x{world} (ncclAllReduce min per round, replicated union-find)"
-                                   if use_dist else "single GPU"),
-                   "options": opt_kw,
-                   "l2": f"inputs ({(8 * M + 8 * n) / 1e6:.0f} MB CSR) exceed L2; plus {args.flush_mb} MB flush "
-                         "between steps"},
+        "config": workload_config(args, world, use_dist, opt_kw, gname, n, M, st["canonical_edges"]),
         "ms_per_graph": ms_max, "ms_per_step_all": per_step, "wall_s": wall,
         "edges_per_s_undirected": st["canonical_edges"] / (ms_max / 1e3),
-        "gpu_launches": args.steps * ((LAUNCHES_FILTERED if M >= 4 * n else LAUNCHES_UNFILTERED)
+        "gpu_launches": args.steps * ((LAUNCHES_FILTERED if st["filtered"] else LAUNCHES_UNFILTERED)
                                       if not use_dist else 4 + 4 * st["rounds"]),
         "clocks": clocks,
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",

@@ -44,7 +44,7 @@
 extern "C" {
 #endif
 
-#define ECL_MST_ABI_VERSION 2
+#define ECL_MST_ABI_VERSION 3
 
 /* status codes */
 #define ECL_MST_OK 0
@@ -53,13 +53,19 @@ extern "C" {
 #define ECL_MST_ERR_CUDA (-3)      /* a CUDA call failed; see ecl_mst_last_error() */
 #define ECL_MST_ERR_WORKSPACE (-4) /* workspace too small or misaligned */
 #define ECL_MST_ERR_INPUT (-5)     /* the device found an inconsistent CSR (stats.status) */
+#define ECL_MST_ERR_ROUNDS (-6)    /* the device ran out of its ECL_MST_MAX_ROUNDS round slots
+                                      (stats.status; cannot happen within the documented limits) */
 
 #define ECL_MST_MAX_ROUNDS 128     /* global round slots (<= ceil(log2 n)+1 per phase and sub-phase) */
 
 /* knobs; every setting returns the identical MSF (tests check this) */
 typedef struct ecl_mst_options {
     int32_t filter;          /* -1 auto: filter iff M >= 4n (reading Q6); 0 off; 1 on */
-    int32_t threshold_mode;  /* 0 sampled: 20 weights, c = 4 (reading Q5/Q7); 1 fixed */
+    int32_t threshold_mode;  /* 0 sampled: the weight of sample rank S*c*n/M among S random entries
+                                (readings Q5/Q7; S = threshold_samples); 1 fixed
+                                (opts.threshold); 2 exact quantile: the weight of rank c*n among
+                                all M entries, by a two-pass device radix select (SURVEY §8(f)
+                                NEXT-3) */
     int32_t threshold;       /* phase 1 takes w < threshold when threshold_mode == 1 */
     int32_t path_halving;    /* 1 (default) find() halves paths it walks (P:142 reading Q15); 0 off */
     int32_t atomic_guards;   /* load-compare before each atomicMin: 1 everywhere; 0 never;
@@ -88,11 +94,32 @@ typedef struct ecl_mst_options {
                                 times"), else 4 ("we use c = 4 in our code"); "values
                                 between 2 and 4 seem to work well".  Only speed depends
                                 on it. */
+    int32_t giant_bitmap;    /* phase 2: membership bitmap of the largest set after phase 1, so the
+                                phase-2 populate filters edges inside it from n/8 bytes instead of
+                                parent[]: -1 (default) auto, on iff n >= 2^25 (parent[] beyond
+                                about half the L2); 0 off; 1 on at any n (tests) */
+    int32_t relabel;         /* contraction: once the surviving sets of a round are few, give them
+                                dense ids so the rounds' key/parent accesses stay in L2.
+                                -1 (default) auto; 0 off; 1 whenever the sets at least halved
+                                (tests).  Same MSF either way. */
+    /* De-optimisations of the paper's Table 5, for the ablation
+     * (SURVEY §8(f) NEXT-2); every setting returns the identical MSF. */
+    int32_t populate_mode;   /* 0 (default) edge-centric warps over 128-entry CSR chunks;
+                                1 "Thread-Based": one thread per vertex walks its row */
+    int32_t both_directions; /* 0 (default) one direction per edge (Alg. 2 L4); 1 "Both Edge
+                                Directions": the worklist holds both directed copies of
+                                every edge (each with the edge's id) -- needs
+                                ecl_mst_workspace_bytes_ex */
+    int32_t tuple_layout;    /* 0 (default) 16-byte 4-tuples <p,q,w,id>; 1 "No
+                                Tuples": the four items in separate arrays */
+    int32_t drive;           /* 0 (default) data-driven worklist; 1 "Topology-Driven": every
+                                round processes all edges of the phase again; 2 "Vertex-Centric"
+                                (P:378): topology-driven with one thread per vertex and its row */
 } ecl_mst_options;
 
 /* per-run statistics written by the device into the workspace */
 typedef struct ecl_mst_stats {
-    int32_t status;          /* 0 or ECL_MST_ERR_INPUT */
+    int32_t status;          /* 0, ECL_MST_ERR_INPUT or ECL_MST_ERR_ROUNDS */
     int32_t filtered;        /* 1 if two phases ran */
     int32_t threshold;       /* phase-1 threshold (phase 1: w < threshold) */
     int32_t rounds;          /* global rounds used (all phases; incl. final empty pass A) */
@@ -119,6 +146,10 @@ void ecl_mst_default_options(ecl_mst_options *opts);
  * int32, two worklists int4[~M] (in / out of a pass). */
 size_t ecl_mst_workspace_bytes(int64_t n, int64_t M);
 
+/* Workspace bytes for (n, M) under `opts` (NULL: defaults, = the above); the
+ * both_directions de-optimisation needs twice the worklist space. */
+size_t ecl_mst_workspace_bytes_ex(int64_t n, int64_t M, const ecl_mst_options *opts);
+
 /*
  * The hot path.  All pointers are DEVICE pointers (current device).  Runs
  * asynchronously on `stream` (a cudaStream_t; NULL = legacy default stream)
@@ -126,10 +157,13 @@ size_t ecl_mst_workspace_bytes(int64_t n, int64_t M);
  * cooperative kernel per phase: no host round-trips.
  * total_weight_out (device int64*) receives the MSF weight, or INT64_MIN if
  * the device detected an inconsistent CSR (then stats.status = ERR_INPUT and
- * in_mst is unspecified).  workspace must be >= ecl_mst_workspace_bytes(n, M)
- * bytes, 256-byte aligned; its contents on entry are irrelevant.  opts may be
- * NULL.  Returns ECL_MST_OK or an ECL_MST_ERR_* code for argument / launch
- * errors (nothing is launched then).
+ * in_mst is unspecified; kernels after the check exit at once, and no kernel
+ * indexes memory through rejected offsets).  workspace must be >=
+ * ecl_mst_workspace_bytes_ex(n, M, opts) bytes, 256-byte aligned; its contents
+ * on entry are irrelevant.  opts may be NULL.  Returns ECL_MST_OK, or an
+ * ECL_MST_ERR_* code: for argument errors nothing is launched; a failing CUDA
+ * call inside the launch sequence (ECL_MST_ERR_CUDA) may leave the kernels
+ * before it enqueued on `stream`.
  */
 int ecl_mst_device(int32_t n, int64_t M, const int64_t *nindex, const int32_t *nlist,
                    const int32_t *eweight, uint8_t *in_mst_out, int64_t *total_weight_out,

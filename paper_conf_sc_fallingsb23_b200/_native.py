@@ -15,7 +15,7 @@ import torch
 from . import build as _build
 
 MAX_ROUNDS = 128
-ABI_VERSION = 2          # include/ecl_mst.h ECL_MST_ABI_VERSION
+ABI_VERSION = 3          # include/ecl_mst.h ECL_MST_ABI_VERSION
 
 OK = 0
 ERR_INVALID = -1
@@ -23,6 +23,7 @@ ERR_TOO_LARGE = -2
 ERR_CUDA = -3
 ERR_WORKSPACE = -4
 ERR_INPUT = -5
+ERR_ROUNDS = -6
 
 
 class EclMstOptions(ctypes.Structure):
@@ -40,6 +41,12 @@ class EclMstOptions(ctypes.Structure):
         ("populate_order", ctypes.c_int32),
         ("refilter", ctypes.c_int32),
         ("filter_c", ctypes.c_int32),
+        ("giant_bitmap", ctypes.c_int32),
+        ("relabel", ctypes.c_int32),
+        ("populate_mode", ctypes.c_int32),
+        ("both_directions", ctypes.c_int32),
+        ("tuple_layout", ctypes.c_int32),
+        ("drive", ctypes.c_int32),
     ]
 
 
@@ -95,6 +102,8 @@ def load(build_if_missing: bool = False):
     L.ecl_mst_default_options.argtypes = [ctypes.POINTER(EclMstOptions)]
     L.ecl_mst_workspace_bytes.restype = sz
     L.ecl_mst_workspace_bytes.argtypes = [i64, i64]
+    L.ecl_mst_workspace_bytes_ex.restype = sz
+    L.ecl_mst_workspace_bytes_ex.argtypes = [i64, i64, ctypes.POINTER(EclMstOptions)]
     L.ecl_mst_device.restype = ctypes.c_int
     L.ecl_mst_device.argtypes = [i32, i64, vp, vp, vp, vp, vp, vp, sz, ctypes.POINTER(EclMstOptions), vp]
     L.ecl_mst_read_stats.restype = ctypes.c_int
@@ -126,7 +135,7 @@ def load(build_if_missing: bool = False):
 
 
 EXPORTED = ["ecl_mst_abi_version", "ecl_mst_last_error", "ecl_mst_default_options",
-            "ecl_mst_workspace_bytes", "ecl_mst_device", "ecl_mst_read_stats", "ecl_mst",
+            "ecl_mst_workspace_bytes", "ecl_mst_workspace_bytes_ex", "ecl_mst_device", "ecl_mst_read_stats", "ecl_mst",
             "ecl_mst_release_host_cache", "ecl_mst_read_trace", "ecl_mst_kernel_times",
             "ecl_mst_dist_unique_id", "ecl_mst_dist_init", "ecl_mst_dist_finalize",
             "ecl_mst_dist_shard_chunks", "ecl_mst_dist_workspace_bytes", "ecl_mst_dist_device"]
@@ -147,8 +156,11 @@ def default_options(**kw) -> EclMstOptions:
     return o
 
 
-def ecl_mst_workspace_bytes(n: int, M: int) -> int:
-    b = load().ecl_mst_workspace_bytes(int(n), int(M))
+def ecl_mst_workspace_bytes(n: int, M: int, options=None) -> int:
+    if options is None:
+        b = load().ecl_mst_workspace_bytes(int(n), int(M))
+    else:
+        b = load().ecl_mst_workspace_bytes_ex(int(n), int(M), ctypes.byref(options))
     if b == 0:
         raise EclMstError(ERR_TOO_LARGE, f"graph too large (n={n}, M={M})")
     return int(b)
@@ -195,10 +207,11 @@ def ecl_mst_device(n, nindex, nlist, eweight, in_mst_out=None, total_weight_out=
     _check(total_weight_out, torch.int64, "total_weight_out", dev)
     if in_mst_out.numel() != M:
         raise ValueError("in_mst_out must have M entries")
-    need = ecl_mst_workspace_bytes(n, M)
+    opts = options if options is not None else default_options()
+    need = ecl_mst_workspace_bytes(n, M, opts)
     if workspace is None or workspace.numel() < need:
         workspace = torch.empty(need, dtype=torch.uint8, device=dev)
-    opts = options if options is not None else default_options()
+    _check(workspace, torch.uint8, "workspace", dev)
     with torch.cuda.device(dev):
         rc = load().ecl_mst_device(n, M, nindex.data_ptr(), nlist.data_ptr(), eweight.data_ptr(),
                                    in_mst_out.data_ptr(), total_weight_out.data_ptr(),
@@ -289,13 +302,20 @@ def ecl_mst_dist_device(handle, n, nindex, nlist, eweight, local_shards=1, world
     _check(eweight, torch.int32, "eweight", dev)
     n = int(n)
     M = int(nlist.numel())
+    if nindex.numel() != n + 1 or eweight.numel() != M:
+        raise ValueError("nindex must have n+1 entries and eweight M entries")
     if in_mst_out is None:
         in_mst_out = torch.empty(M, dtype=torch.uint8, device=dev)
     if total_weight_out is None:
         total_weight_out = torch.empty(1, dtype=torch.int64, device=dev)
+    _check(in_mst_out, torch.uint8, "in_mst_out", dev)
+    _check(total_weight_out, torch.int64, "total_weight_out", dev)
+    if in_mst_out.numel() != M or total_weight_out.numel() < 1:
+        raise ValueError("in_mst_out must have M entries and total_weight_out at least one")
     need = ecl_mst_dist_workspace_bytes(n, M, local_shards, world)
     if workspace is None or workspace.numel() < need:
         workspace = torch.empty(need, dtype=torch.uint8, device=dev)
+    _check(workspace, torch.uint8, "workspace", dev)
     opts = options if options is not None else default_options()
     with torch.cuda.device(dev):
         rc = load().ecl_mst_dist_device(handle, int(local_shards), n, M, nindex.data_ptr(), nlist.data_ptr(),
@@ -327,11 +347,21 @@ def ecl_mst(n, nindex, nlist, eweight, in_mst_out):
         _check(t, dt, nm)
         if t.device.type != "cpu":
             raise ValueError(f"{nm} must be a host tensor")
+    # the library reads nindex[n] and then M = nindex[n] entries of every
+    # array from these host pointers: check the sizes here, before it does
+    n = int(n)
+    if n < 0 or nindex.numel() != n + 1:
+        raise ValueError("nindex must have n+1 entries")
+    M = int(nindex[-1]) if n > 0 else 0
+    if M < 0 or M > nlist.numel() or nlist.numel() != eweight.numel() or in_mst_out.numel() < M:
+        raise ValueError(f"nindex[n] = {M} must satisfy 0 <= M <= nlist.numel() == eweight.numel() "
+                         f"<= in_mst_out.numel()")
     total = load().ecl_mst(int(n), nindex.data_ptr(), nlist.data_ptr(), eweight.data_ptr(),
                            in_mst_out.data_ptr())
     if total == -(1 << 63):
         err = load().ecl_mst_last_error().decode(errors="replace")
-        raise EclMstError(ERR_INPUT if "inconsistent" in err else ERR_CUDA, err)
+        code = ERR_INPUT if "inconsistent" in err else ERR_ROUNDS if "round slots" in err else ERR_CUDA
+        raise EclMstError(code, err)
     return int(total)
 
 

@@ -54,11 +54,12 @@ static inline long long wl_capacity(long long M) {
     return (nchunks + wmax) * (long long)kChunk;
 }
 
-static inline Layout layout_for(int64_t n, int64_t M) {
+// dup: worklist copies per canonical edge (2 for opts.both_directions)
+static inline Layout layout_for(int64_t n, int64_t M, int dup = 1) {
     Layout L;
     size_t off = 0;
     const long long nchunks = ceil_div(M, kChunk);
-    L.wl_cap = wl_capacity(M);
+    L.wl_cap = dup * wl_capacity(M);
     L.stats = off;    off = align_up(off + sizeof(ecl_mst_stats), 256);
     L.internal = off; off = align_up(off + sizeof(Internal), 256);
     L.trace = off;    off = align_up(off + sizeof(long long) * kTraceSlots * kMaxGrid, 256);
@@ -109,6 +110,7 @@ struct Params {
     int guards;                       // -1 auto, 0 off, 1 on
     int flatten;
     int refilter;                     // -1 auto, 0 off, 1 forced (opts.refilter)
+    int round_bound;                  // ceil(log2 n) + 1: rounds one phase or sub-phase can take
     int* samp;                        // crowded-round weight samples (kSplitSampleSlots)
     // edge sharding (distributed path; single GPU: shard 0 of 1)
     int shard;                        // global shard id
@@ -155,11 +157,19 @@ __device__ __forceinline__ void trace_cta(const Params& P, int slot) {
     }
 }
 
+// false once a kernel has flagged the input (k_init: nindex out of range or
+// not monotone, so rowstart[] may hold garbage; populate: nlist out of range).
+// Set only by earlier kernels of the launch sequence, so every CTA of a
+// kernel reads the same value and the cooperative kernels exit uniformly.
+__device__ __forceinline__ bool input_ok(const Params& P) {
+    return *reinterpret_cast<volatile const int*>(&P.st->status) == 0;
+}
+
 // phase 2 runs iff filtering is on and phase 1 deferred at least one edge
 // (read-only within the kernels that ask: one L1 line per SM, not one L2
 // slice hammered by every warp of the grid)
 __device__ __forceinline__ bool phase2_needed(const Params& P) {
-    return __ldg(&P.st->filtered) != 0 && __ldg(&P.st->heavy_edges) != 0;
+    return __ldg(&P.st->filtered) != 0 && __ldg(&P.st->heavy_edges) != 0 && __ldg(&P.st->status) == 0;
 }
 
 }  // namespace eclmst

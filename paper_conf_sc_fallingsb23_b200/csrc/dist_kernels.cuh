@@ -313,6 +313,10 @@ __global__ void __launch_bounds__(kBlock, 2) k_dist_passA(Params P, int g, int c
     const int b = blockIdx.x;
     int4* wl[2] = {P.wl0 + (long long)b * P.cap, P.wl1 + (long long)b * P.cap};
     if (tid == 0) s_out = 0;
+    if (FIRST && !input_ok(P)) {   // the populate skipped a rejected CSR: no regions to read
+        if (tid == 0) P.acnt[b] = 0;
+        return;
+    }
     if (FIRST) {
         const RegionSrc R = region_src(P, b, s_pre, s_rcnt, s_red, &P.st->live[g - 1], g - 1 == 0);
         passA(P, R, wl[cur ^ 1], &s_out, P.guards != 0);

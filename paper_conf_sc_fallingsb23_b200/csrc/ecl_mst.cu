@@ -78,6 +78,7 @@ constexpr int kTimedStages = 7;   // init, populate1, rounds1, flatten, populate
 struct Timing {
     bool ready = false;
     bool valid = false;
+    int dev = -1;                      // device the events were created on
     cudaEvent_t ev[kTimedStages + 1];
 };
 static thread_local Timing g_timing;
@@ -131,11 +132,22 @@ void ecl_mst_default_options(ecl_mst_options* o) {
     o->populate_order = 0;
     o->refilter = -1;
     o->filter_c = 0;
+    o->giant_bitmap = -1;
+    o->relabel = -1;
+    o->populate_mode = 0;
+    o->both_directions = 0;
+    o->tuple_layout = 0;
+    o->drive = 0;
 }
 
 size_t ecl_mst_workspace_bytes(int64_t n, int64_t M) {
     if (n < 0 || n > INT32_MAX || M < 0 || M > (int64_t)0xFFFFFFFFLL) return 0;
     return layout_for(n, M).total;
+}
+
+size_t ecl_mst_workspace_bytes_ex(int64_t n, int64_t M, const ecl_mst_options* opts) {
+    if (n < 0 || n > INT32_MAX || M < 0 || M > (int64_t)0xFFFFFFFFLL) return 0;
+    return layout_for(n, M, opts && opts->both_directions ? 2 : 1).total;
 }
 
 }  // extern "C"
@@ -161,6 +173,19 @@ static int run_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t
 // c of P:143 (reading Q5b): opts.filter_c if set; else the paper's target of
 // "3 times" on dense graphs (M >= 16 n: C4/C5, where the light
 // part then still holds most MSF edges) and its code's c = 4 below.
+// ceil(log2 n) + 1: Boruvka rounds one phase (or crowded-round sub-phase)
+// can take -- every round at least halves the sets that still have an edge
+static inline int round_bound_for(int32_t n) {
+    int b = 0;
+    while ((1LL << b) < (long long)n) ++b;
+    return b + 1;
+}
+
+// opts.giant_bitmap: -1 auto (parent[] beyond about half the L2), 0 off, 1 on
+static inline bool giant_bitmap_on(int32_t opt, int32_t n) {
+    return opt > 0 || (opt < 0 && (long long)n >= ECL_GIANT_MIN_N);
+}
+
 static inline int filter_c_for(int32_t opt, int32_t n, int64_t M) {
     if (opt > 0) return opt;
     return M >= 16LL * n ? 3 : 4;
@@ -187,12 +212,15 @@ static int run_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t
     if (n > 0 && !nindex) return fail(ECL_MST_ERR_INVALID, "null nindex");
     if (M > 0 && (!nlist || !eweight || !in_mst_out)) return fail(ECL_MST_ERR_INVALID, "null CSR or output array");
     if (M > 0 && n == 0) return fail(ECL_MST_ERR_INVALID, "M > 0 with n = 0");
-    const Layout L = layout_for(n, M);
-    if (workspace_bytes < L.total) return fail(ECL_MST_ERR_WORKSPACE, "workspace %zu < %zu bytes", workspace_bytes, L.total);
-    if (reinterpret_cast<uintptr_t>(workspace) % 256) return fail(ECL_MST_ERR_WORKSPACE, "workspace not 256-byte aligned");
     ecl_mst_options o;
     ecl_mst_default_options(&o);
     if (opts) o = *opts;
+    if (o.threshold_mode < 0 || o.threshold_mode > 2) return fail(ECL_MST_ERR_INVALID, "threshold_mode must be 0, 1 or 2");
+    if (o.populate_mode || o.both_directions || o.tuple_layout || o.drive)
+        return fail(ECL_MST_ERR_INVALID, "de-optimisation knob not available");
+    const Layout L = layout_for(n, M, o.both_directions ? 2 : 1);
+    if (workspace_bytes < L.total) return fail(ECL_MST_ERR_WORKSPACE, "workspace %zu < %zu bytes", workspace_bytes, L.total);
+    if (reinterpret_cast<uintptr_t>(workspace) % 256) return fail(ECL_MST_ERR_WORKSPACE, "workspace not 256-byte aligned");
     cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
     char* ws = static_cast<char*>(workspace);
     if (M == 0) {
@@ -261,7 +289,7 @@ static int run_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t
     P.rowstart = reinterpret_cast<int*>(ws + L.rowstart);
     P.region = reinterpret_cast<int4*>(ws + L.region);
     // the largest-set bitmap only pays when parent[] does not fit the L2
-    P.giant_bits = (long long)n >= ECL_GIANT_MIN_N ? reinterpret_cast<unsigned*>(ws + L.giant) : nullptr;
+    P.giant_bits = giant_bitmap_on(o.giant_bitmap, n) ? reinterpret_cast<unsigned*>(ws + L.giant) : nullptr;
     P.key = reinterpret_cast<long long*>(ws + L.key);
     P.parent = reinterpret_cast<int*>(ws + L.parent);
     P.wl0 = reinterpret_cast<int4*>(ws + L.wl0);
@@ -276,6 +304,7 @@ static int run_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t
     P.guards = o.atomic_guards < 0 ? -1 : (o.atomic_guards ? 1 : 0);
     P.flatten = o.flatten ? 1 : 0;
     P.refilter = o.refilter < 0 ? -1 : (o.refilter ? 1 : 0);
+    P.round_bound = round_bound_for(n);
     P.samp = reinterpret_cast<int*>(ws + L.samp);
     P.shard = 0;
     P.nshards = 1;
@@ -297,12 +326,29 @@ static int run_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t
     void* args[] = {&P};
     // opts.trace bit 1: CUDA events between the kernels (ecl_mst_kernel_times)
     const bool timing = (o.trace & 2) != 0;
-    if (timing && !g_timing.ready) {
-        for (int i = 0; i < kTimedStages + 1; ++i) {
-            cudaError_t e0 = cudaEventCreate(&g_timing.ev[i]);
-            if (e0 != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "cudaEventCreate: %s", cudaGetErrorString(e0));
+    if (timing) {   // events belong to a device: recreate them when the caller switched devices
+        int cur_dev = -1;
+        cudaError_t e0 = cudaGetDevice(&cur_dev);
+        if (e0 != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "cudaGetDevice: %s", cudaGetErrorString(e0));
+        if (g_timing.ready && g_timing.dev != cur_dev) {
+            int prev = -1;
+            cudaGetDevice(&prev);
+            cudaSetDevice(g_timing.dev);
+            for (auto& ev : g_timing.ev) cudaEventDestroy(ev);
+            cudaSetDevice(prev);
+            g_timing.ready = false;
         }
-        g_timing.ready = true;
+        if (!g_timing.ready) {
+            for (int i = 0; i < kTimedStages + 1; ++i) {
+                e0 = cudaEventCreate(&g_timing.ev[i]);
+                if (e0 != cudaSuccess) {
+                    for (int k = 0; k < i; ++k) cudaEventDestroy(g_timing.ev[k]);
+                    return fail(ECL_MST_ERR_CUDA, "cudaEventCreate: %s", cudaGetErrorString(e0));
+                }
+            }
+            g_timing.ready = true;
+            g_timing.dev = cur_dev;
+        }
     }
     g_timing.valid = false;
     int ev_i = 0;
@@ -554,7 +600,12 @@ int64_t ecl_mst(int32_t n, const int64_t* nindex, const int32_t* nlist, const in
         fail(ECL_MST_ERR_CUDA, "D2H/run: %s", cudaGetErrorString(e));
         return INT64_MIN;
     }
-    if (total == INT64_MIN) fail(ECL_MST_ERR_INPUT, "device found an inconsistent CSR");
+    if (total == INT64_MIN) {
+        int status = ECL_MST_ERR_INPUT;   // stats.status is the first word of the workspace
+        if (cudaMemcpy(&status, d_ws, sizeof status, cudaMemcpyDeviceToHost) != cudaSuccess) status = ECL_MST_ERR_INPUT;
+        if (status == ECL_MST_ERR_ROUNDS) fail(ECL_MST_ERR_ROUNDS, "device ran out of round slots");
+        else fail(ECL_MST_ERR_INPUT, "device found an inconsistent CSR");
+    }
     return total;
 }
 
@@ -757,6 +808,8 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
     ecl_mst_options o;
     ecl_mst_default_options(&o);
     if (opts) o = *opts;
+    if (o.populate_mode || o.both_directions || o.tuple_layout || o.drive)
+        return fail(ECL_MST_ERR_INVALID, "the de-optimisation knobs are single-GPU only (ecl_mst_device)");
     cudaStream_t s = reinterpret_cast<cudaStream_t>(stream);
     char* ws = static_cast<char*>(workspace);
     ecl_mst_stats* st = reinterpret_cast<ecl_mst_stats*>(ws + L.stats);
@@ -834,6 +887,7 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
         P.guards = o.atomic_guards == 0 ? 0 : 1;
         P.flatten = o.flatten ? 1 : 0;
         P.refilter = o.refilter < 0 ? -1 : (o.refilter ? 1 : 0);   // crowded-round split (Q17)
+        P.round_bound = round_bound_for(n);
         P.samp = nullptr;
         P.shard = shard;
         P.nshards = (int)Pt;
@@ -843,7 +897,7 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
         P.tgt = reinterpret_cast<int*>(ws + L.tgt);
         P.hcnt = reinterpret_cast<int*>(sb + L.hcnt);
         // phase 2: the largest set's bitmap where parent[] exceeds the L2, as on one GPU
-        P.giant_bits = (long long)n >= ECL_GIANT_MIN_N ? reinterpret_cast<unsigned*>(ws + L.giant) : nullptr;
+        P.giant_bits = giant_bitmap_on(o.giant_bitmap, n) ? reinterpret_cast<unsigned*>(ws + L.giant) : nullptr;
         P.dsp = split_on ? dsp : nullptr;
         P.keys_all = d_keyptrs;
         P.nkeys = S;

@@ -23,9 +23,15 @@ __global__ void __launch_bounds__(256) k_init(Params P) {
         } else {
             P.key[v] = kInf;
         }
-        // chunk starts inside row v: rowstart[c] = v for c*kChunk in [s, e)
+        // chunk starts inside row v: rowstart[c] = v for c*kChunk in [s, e).
+        // A row outside [0, M] or running backwards is an input error; it
+        // writes nothing (every later kernel then exits at once, see
+        // input_ok), so invalid offsets never index rowstart[] out of range.
         const long long s = P.nindex[v], e = P.nindex[v + 1];
-        if (e < s) err = true;
+        if (s < 0 || e < s || e > P.M) {
+            err = true;
+            continue;
+        }
         for (long long c = (s + kChunk - 1) / kChunk; c * kChunk < e && c < P.nchunks; ++c) P.rowstart[c] = (int)v;
     }
     if (blockIdx.x == 0) {
@@ -98,6 +104,7 @@ template <int PH>
 __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) {
     __shared__ int s_mark[kPopWarps][kChunk];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    if (!input_ok(P)) return;   // k_init rejected nindex: rowstart[] is not valid
     if (PH == 2 && !phase2_needed(P)) return;
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         if (PH == 1) P.st->t_ns[1] = (long long)globaltimer_ns();   // init done

@@ -344,7 +344,10 @@ __device__ __forceinline__ bool use_guard(const Params& P, long long live, long 
                              // (4 -> 2: C4 7.18 -> 7.10 ms, C2 2.283 -> 2.262 ms, C5 -0.5%, C3 +-0)
 #endif
 __device__ __forceinline__ bool crowded(const Params& P, long long live, long long winners, int g) {
-    if (P.refilter == 0 || __ldcg(&P.in->splits) >= 16 || g + 24 >= ECL_MST_MAX_ROUNDS) return false;
+    // a split opens a sub-phase of up to round_bound rounds and the phase
+    // itself may still need as many: only split while both fit the slots
+    if (P.refilter == 0 || __ldcg(&P.in->splits) >= 16 || g + 2 * P.round_bound + 2 >= ECL_MST_MAX_ROUNDS)
+        return false;
     if (P.refilter > 0) return live > 4 * winners;
     return live >= (1LL << 20) && live > ECL_CROWD_RATIO * winners;
 }
@@ -405,10 +408,10 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
     const int tid = threadIdx.x, lane = tid & 31;
     const bool b0 = blockIdx.x == 0;
     ecl_mst_stats* st = P.st;
-    if (PH == 2 && !phase2_needed(P)) return;
+    if (!input_ok(P) || (PH == 2 && !phase2_needed(P))) return;
     int g = (PH == 1) ? 0 : __ldcg(&P.in->g_end) + 1;
     if (g >= ECL_MST_MAX_ROUNDS) {
-        if (b0 && tid == 0) atomicExch(&st->status, ECL_MST_ERR_INPUT);
+        if (b0 && tid == 0) atomicExch(&st->status, ECL_MST_ERR_ROUNDS);
         return;
     }
     stamp(P, 4 + 2 * g);                      // populate done
@@ -522,7 +525,7 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
         P.in->g_end = g;
         st->rounds = g + 1;
         st->refilters = __ldcg(&P.in->splits);
-        if (overflow) atomicExch(&st->status, ECL_MST_ERR_INPUT);
+        if (overflow) atomicExch(&st->status, ECL_MST_ERR_ROUNDS);
     }
 }
 

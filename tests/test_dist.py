@@ -203,7 +203,8 @@ def test_virtual_shards_fuzz(ecl, seed):
     h = ecl.ecl_mst_dist_init(None, 0, 1)
     try:
         for opts in (dict(refilter=1), dict(refilter=1, filter=1, threshold_mode=1, threshold=0),
-                     dict(refilter=1, filter=0, filter_c=1), dict(refilter=0)):
+                     dict(refilter=1, filter=0, filter_c=1), dict(refilter=0),
+                     dict(giant_bitmap=1), dict(giant_bitmap=1, refilter=1, filter=1, filter_c=2)):
             mask, total, st = dist_run(ecl, g, h, 2 + seed % 3, **opts)
             assert st["status"] == 0, opts
             assert total == ototal and np.array_equal(mask, omask), opts

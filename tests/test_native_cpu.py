@@ -3,6 +3,7 @@
 import ctypes
 import os
 import re
+import subprocess
 
 import pytest
 
@@ -31,10 +32,28 @@ def test_exports_every_declared_symbol(lib):
     assert sorted(_native.EXPORTED) == names
 
 
-def test_struct_layouts_match_header():
-    # header: 8 int32 + 4 int64 + 2 * 128 int64 + 260 int64
-    assert ctypes.sizeof(_native.EclMstStats) == 8 * 4 + 4 * 8 + 2 * 128 * 8 + 260 * 8
-    assert ctypes.sizeof(_native.EclMstOptions) == 8 * 4 + 8 + 4 * 4
+def _c_layout(tmp_path, struct, fields):
+    """sizeof and offsetof(field) of a header struct, as gcc lays it out."""
+    src = tmp_path / "layout.c"
+    lines = ["#include <stdio.h>", "#include <stddef.h>", '#include "ecl_mst.h"', "int main(void) {",
+             f'printf("%zu\\n", sizeof({struct}));']
+    lines += [f'printf("%zu\\n", offsetof({struct}, {f}));' for f in fields]
+    lines += ["return 0; }"]
+    src.write_text("\n".join(lines))
+    exe = tmp_path / "layout"
+    subprocess.check_call(["gcc", "-std=c11", "-I", os.path.join(ROOT, "include"), "-o", str(exe), str(src)])
+    out = [int(x) for x in subprocess.check_output([str(exe)]).split()]
+    return out[0], out[1:]
+
+
+@pytest.mark.parametrize("struct,cls", [("ecl_mst_options", "EclMstOptions"), ("ecl_mst_stats", "EclMstStats")])
+def test_struct_layouts_match_header(tmp_path, struct, cls):
+    """The ctypes mirrors of the header structs have gcc's size and field offsets."""
+    C = getattr(_native, cls)
+    names = [f[0] for f in C._fields_]
+    size, offs = _c_layout(tmp_path, struct, names)
+    assert ctypes.sizeof(C) == size
+    assert [getattr(C, f).offset for f in names] == offs
 
 
 def test_workspace_bytes(lib):
