@@ -127,6 +127,8 @@ typedef struct ecl_mst_stats {
     int32_t grid;            /* CTAs of the persistent launch */
     int32_t block;           /* threads per CTA */
     int32_t refilters;       /* crowded-round splits taken (opts.refilter); each adds one sub-phase */
+    int32_t relabels;        /* contraction levels opened (opts.relabel) */
+    int32_t reserved;
     int64_t total_weight;
     int64_t msf_edges;
     int64_t canonical_edges; /* |E| = #{j : u < nlist[j]} */

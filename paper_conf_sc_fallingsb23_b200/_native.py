@@ -60,6 +60,8 @@ class EclMstStats(ctypes.Structure):
         ("grid", ctypes.c_int32),
         ("block", ctypes.c_int32),
         ("refilters", ctypes.c_int32),
+        ("relabels", ctypes.c_int32),
+        ("reserved", ctypes.c_int32),
         ("total_weight", ctypes.c_int64),
         ("msf_edges", ctypes.c_int64),
         ("canonical_edges", ctypes.c_int64),
@@ -233,7 +235,7 @@ def ecl_mst_read_stats(workspace, stream=None) -> dict:
     return {
         "status": st.status, "filtered": bool(st.filtered), "threshold": st.threshold,
         "rounds": st.rounds, "phase2_round": st.phase2_round, "grid": st.grid, "block": st.block,
-        "refilters": st.refilters,
+        "refilters": st.refilters, "relabels": st.relabels,
         "total_weight": st.total_weight, "msf_edges": st.msf_edges,
         "canonical_edges": st.canonical_edges, "heavy_edges": st.heavy_edges,
         "live": list(st.live[:R]), "winners": list(st.winners[:R]),

@@ -25,6 +25,8 @@ constexpr int kMaxSamples = 4096;              // threshold sample size cap
 constexpr int kStagePieces = 8;                // host path: CSR pieces uploaded under the populate
 constexpr int kSplitSamples = 512;             // crowded-round threshold: about this many samples
 constexpr int kSplitSampleSlots = 1024;        // sample slots (max(1, 512 / G) per CTA, first CTAs)
+constexpr int kQBins = 2048;                   // exact-quantile radix select: 11 + 11 + 10 bits
+constexpr int kMaxLevels = 24;                 // relabel: contraction levels (level 0 = the vertices)
 static_assert(kMaxGrid == ECL_MST_TRACE_CTAS, "trace layout");
 
 struct Internal {
@@ -35,10 +37,23 @@ struct Internal {
     int g_end;                         // last global round of the finished phase
     int giant;                         // root of the largest set after phase 1 (-1: none)
     int splits;                        // crowded-round splits taken so far (all phases)
+    unsigned q_prefix;                 // exact-quantile threshold: bits of the order key fixed so far
+    long long q_rank;                  // ... and the rank still to find below that prefix
+    // contraction levels (opts.relabel).  Set ids are absolute indices into
+    // parent[] / key[] (2n slots each): level 0 (the vertices) is [0, n), each
+    // later level the next free range of [n, 2n) (levels at least halve, so
+    // they fit).  Levels below the open one are closed: every root stores
+    // ~label, its id in the next level.  Written by k_rounds<1> at exit, read
+    // by the flatten and by k_rounds<2>.
+    int nlev;                          // closed levels
+    long long lv_base;                 // first id of the open level
+    long long lv_size;                 // ids in the open level
+    long long lv_roots;                // roots in the open level
+    long long lv_next;                 // first id of the next level
 };
 
 struct Layout {
-    size_t stats, internal, trace, rowstart, region, giant, samp, key, parent, wl0, wl1, total;
+    size_t stats, internal, trace, rowstart, region, giant, samp, qhist, lvcnt, key, parent, setid, wl0, wl1, total;
     long long wl_cap;                  // tuples per worklist buffer
 };
 
@@ -67,8 +82,12 @@ static inline Layout layout_for(int64_t n, int64_t M, int dup = 1) {
     L.region = off;   off = align_up(off + sizeof(int4) * (size_t)kMaxPopWarps, 256);
     L.giant = off;    off = align_up(off + sizeof(unsigned) * (size_t)((n + 31) / 32 + 1), 256);
     L.samp = off;     off = align_up(off + sizeof(int) * (size_t)kSplitSampleSlots, 256);
-    L.key = off;      off = align_up(off + sizeof(long long) * (size_t)n, 256);
-    L.parent = off;   off = align_up(off + sizeof(int) * (size_t)n, 256);
+    L.qhist = off;    off = align_up(off + sizeof(unsigned long long) * (size_t)kQBins, 256);
+    L.lvcnt = off;    off = align_up(off + sizeof(int) * (size_t)kMaxGrid, 256);
+    // key / parent: 2n slots, the vertices plus the contraction levels (Internal)
+    L.key = off;      off = align_up(off + sizeof(long long) * (size_t)(2 * n), 256);
+    L.parent = off;   off = align_up(off + sizeof(int) * (size_t)(2 * n), 256);
+    L.setid = off;    off = align_up(off + sizeof(int) * (size_t)n, 256);
     L.wl0 = off;      off = align_up(off + sizeof(int4) * (size_t)L.wl_cap, 256);
     L.wl1 = off;      off = align_up(off + sizeof(int4) * (size_t)L.wl_cap, 256);
     L.total = off;
@@ -112,6 +131,10 @@ struct Params {
     int refilter;                     // -1 auto, 0 off, 1 forced (opts.refilter)
     int round_bound;                  // ceil(log2 n) + 1: rounds one phase or sub-phase can take
     int* samp;                        // crowded-round weight samples (kSplitSampleSlots)
+    unsigned long long* qhist;        // exact-quantile histogram (kQBins)
+    int relabel;                      // -1 auto, 0 off, 1 whenever the sets at least halved (opts.relabel)
+    int* lvcnt;                       // per-CTA root counts of a relabel (kMaxGrid)
+    int* setid;                       // set of every vertex after phase 1 (k_flatten), read by populate 2
     // edge sharding (distributed path; single GPU: shard 0 of 1)
     int shard;                        // global shard id
     int nshards;                      // total shards
@@ -143,6 +166,7 @@ __device__ __forceinline__ DS ds_of(const Params& P) {
     D.key = P.key;
     return D;
 }
+
 
 __device__ __forceinline__ void stamp(const Params& P, int slot) {
     if (blockIdx.x == 0 && threadIdx.x == 0 && slot < kTraceSlots)

@@ -77,6 +77,21 @@ __device__ __forceinline__ int find_root(const DS& D, int x, bool halving) {
     return find_from(D, x, __ldca(D.par(x)), halving);
 }
 
+// find() in a CLOSED contraction level (opts.relabel): every root r stores
+// ~label(r), its id in the next level, so the walk ends at the first negative
+// entry and returns that label.  Halving re-points x to its grandparent as
+// above (only non-negative ancestors are ever stored).
+__device__ __forceinline__ int find_label_from(int* par, int x, int px, bool halving) {
+    while (px >= 0) {
+        const int ppx = __ldca(par + px);
+        if (ppx < 0) return ~ppx;
+        if (halving) par[x] = ppx;
+        x = ppx;
+        px = __ldca(par + x);
+    }
+    return ~px;
+}
+
 // 64-bit atomicMin (L20-21) with the paper's optional guard: a plain
 // load first, skipping the atomic when it cannot lower the slot.  The guard
 // may read through L1: slots only decrease during a pass, so a stale value is

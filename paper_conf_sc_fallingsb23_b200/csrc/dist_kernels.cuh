@@ -319,7 +319,7 @@ __global__ void __launch_bounds__(kBlock, 2) k_dist_passA(Params P, int g, int c
     }
     if (FIRST) {
         const RegionSrc R = region_src(P, b, s_pre, s_rcnt, s_red, &P.st->live[g - 1], g - 1 == 0);
-        passA(P, R, wl[cur ^ 1], &s_out, P.guards != 0);
+        passA(P, ds_of(P), R, wl[cur ^ 1], &s_out, P.guards != 0);
     } else {
         // a crowded-round split (decided by k_dist_split_decide): light
         // tuples to the front of the output arena, the rest deferred to its
@@ -330,11 +330,11 @@ __global__ void __launch_bounds__(kBlock, 2) k_dist_passA(Params P, int g, int c
         __syncthreads();
         const CompactSrc S = compact_src(wl[cur], P.acnt[b]);
         if (T != INT_MAX) {
-            passA<true>(P, S, wl[cur ^ 1], &s_out, P.guards != 0, T, wl[cur ^ 1] + P.cap, &s_def);
+            passA<true>(P, ds_of(P), S, wl[cur ^ 1], &s_out, P.guards != 0, T, wl[cur ^ 1] + P.cap, &s_def);
             __syncthreads();
             if (tid == 0) P.hcnt[b] = s_def;
         } else {
-            passA(P, S, wl[cur ^ 1], &s_out, P.guards != 0);
+            passA(P, ds_of(P), S, wl[cur ^ 1], &s_out, P.guards != 0);
         }
     }
     __syncthreads();
@@ -355,7 +355,7 @@ __global__ void __launch_bounds__(kBlock, 2) k_dist_drain(Params P, int g, int h
     if (tid == 0) s_out = 0;
     __syncthreads();
     const int h = P.hcnt[b];
-    passA(P, compact_src(wl[hb] + P.cap - h, h), wl[hb ^ 1], &s_out, true);
+    passA(P, ds_of(P), compact_src(wl[hb] + P.cap - h, h), wl[hb ^ 1], &s_out, true);
     __syncthreads();
     if (tid == 0) {
         P.acnt[b] = s_out;

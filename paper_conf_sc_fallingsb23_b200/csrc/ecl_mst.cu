@@ -186,6 +186,20 @@ static inline bool giant_bitmap_on(int32_t opt, int32_t n) {
     return opt > 0 || (opt < 0 && (long long)n >= ECL_GIANT_MIN_N);
 }
 
+// threshold_mode 2: the three radix-select passes after k_init (the kernels
+// return at once when the graph is not filtered)
+static cudaError_t launch_quantile(const Params& P, const DevInfo& di, cudaStream_t s) {
+    if (P.threshold_mode != 2 || !(P.filter_mode > 0 || (P.filter_mode < 0 && P.M >= 4LL * P.n))) return cudaSuccess;
+    const unsigned hb = (unsigned)std::max<long long>(1, std::min<long long>(ceil_div(P.M / 4 + 1, 256), (long long)di.sms * 8));
+    k_qhist<1><<<hb, 256, 0, s>>>(P);
+    k_qselect<1><<<1, 1024, 0, s>>>(P);
+    k_qhist<2><<<hb, 256, 0, s>>>(P);
+    k_qselect<2><<<1, 1024, 0, s>>>(P);
+    k_qhist<3><<<hb, 256, 0, s>>>(P);
+    k_qselect<3><<<1, 1024, 0, s>>>(P);
+    return cudaGetLastError();
+}
+
 static inline int filter_c_for(int32_t opt, int32_t n, int64_t M) {
     if (opt > 0) return opt;
     return M >= 16LL * n ? 3 : 4;
@@ -306,6 +320,12 @@ static int run_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t
     P.refilter = o.refilter < 0 ? -1 : (o.refilter ? 1 : 0);
     P.round_bound = round_bound_for(n);
     P.samp = reinterpret_cast<int*>(ws + L.samp);
+    P.qhist = reinterpret_cast<unsigned long long*>(ws + L.qhist);
+    // contraction needs the flatten (phase 2 then reads every vertex's set from setid)
+    // (absolute level ids up to 2n must fit int32)
+    P.relabel = (o.flatten && (long long)n <= (1LL << 30)) ? (o.relabel < 0 ? -1 : (o.relabel ? 1 : 0)) : 0;
+    P.lvcnt = reinterpret_cast<int*>(ws + L.lvcnt);
+    P.setid = reinterpret_cast<int*>(ws + L.setid);
     P.shard = 0;
     P.nshards = 1;
     P.nlocal = nchunks;
@@ -364,7 +384,8 @@ static int run_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t
     if (stg) {
         // nindex first (k_init needs all of it), and eweight too when the
         // threshold samples it; then the pieces of nlist (and eweight)
-        const bool sampled = (P.filter_mode > 0 || (P.filter_mode < 0 && M >= 4LL * n)) && P.threshold_mode == 0;
+        const bool sampled = (P.filter_mode > 0 || (P.filter_mode < 0 && M >= 4LL * n)) &&
+                             (P.threshold_mode == 0 || P.threshold_mode == 2);
         e = cudaMemcpyAsync(const_cast<int64_t*>(nindex), stg->h_idx, sizeof(int64_t) * ((size_t)n + 1),
                             cudaMemcpyHostToDevice, stg->copy);
         if (e == cudaSuccess && sampled)
@@ -395,6 +416,7 @@ static int run_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t
         k_init<<<flat_blocks, 256, 0, s>>>(P);
         e = cudaGetLastError();
     }
+    if (e == cudaSuccess) e = launch_quantile(P, di, s);
     if (e == cudaSuccess) e = mark();
     if (e == cudaSuccess) {
         if (staged) {   // one launch per piece, each after its piece has landed
@@ -674,7 +696,8 @@ static void release(DistHandle* h) {
 }
 
 struct DistLayout {
-    size_t stats, internal, rowstart, parent, tgt, keyptrs, rl0, rl1, rbuf, keep, bcnt, dsplit, giant, shard0, shard_bytes, total;
+    size_t stats, internal, rowstart, parent, tgt, keyptrs, rl0, rl1, rbuf, keep, bcnt, dsplit, giant, qhist, setid,
+        shard0, shard_bytes, total;
     size_t region, acnt, hcnt, key, wl0, wl1;   // offsets inside one shard block
     long long wl_cap, nlocal_max;
 };
@@ -700,6 +723,8 @@ static inline DistLayout dist_layout(int64_t n, int64_t M, int S, int world) {
     L.bcnt = off;     off = align_up(off + sizeof(int) * (size_t)kCompactGridMax, 256);
     L.dsplit = off;   off = align_up(off + sizeof(DistSplit), 256);
     L.giant = off;    off = align_up(off + sizeof(unsigned) * (size_t)((n + 31) / 32 + 1), 256);   // largest-set bitmap
+    L.qhist = off;    off = align_up(off + sizeof(unsigned long long) * (size_t)kQBins, 256);
+    L.setid = off;    off = align_up(off + sizeof(int) * (size_t)n, 256);
     size_t so = 0;
     L.region = so; so = align_up(so + sizeof(int4) * (size_t)kMaxPopWarps, 256);
     L.acnt = so;   so = align_up(so + sizeof(int) * (size_t)kMaxGrid, 256);
@@ -889,6 +914,10 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
         P.refilter = o.refilter < 0 ? -1 : (o.refilter ? 1 : 0);   // crowded-round split (Q17)
         P.round_bound = round_bound_for(n);
         P.samp = nullptr;
+        P.qhist = reinterpret_cast<unsigned long long*>(ws + L.qhist);
+        P.relabel = 0;   // (the replicated union-find stays on vertex ids)
+        P.lvcnt = nullptr;
+        P.setid = reinterpret_cast<int*>(ws + L.setid);
         P.shard = shard;
         P.nshards = (int)Pt;
         P.nlocal = nlocal;
@@ -930,6 +959,8 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
     if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "memset: %s", cudaGetErrorString(e));
     k_init<<<vblocks, 256, 0, s>>>(P0);
     if ((rc = check("k_init"))) return rc;
+    e = launch_quantile(P0, di, s);   // every rank holds the full CSR: the same threshold everywhere
+    if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "quantile: %s", cudaGetErrorString(e));
     int g = 0;
     int* const rlist[2] = {reinterpret_cast<int*>(ws + L.rl0), reinterpret_cast<int*>(ws + L.rl1)};
     unsigned char* const rkeep = reinterpret_cast<unsigned char*>(ws + L.keep);

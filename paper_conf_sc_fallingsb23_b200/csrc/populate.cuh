@@ -76,9 +76,98 @@ __global__ void __launch_bounds__(256) k_init(Params P) {
             P.in->done = 0;
             P.in->giant = -1;
             P.in->splits = 0;
+            // exact quantile (threshold_mode 2): the entry of rank c|V| (0-based,
+            // at most M - 1) among all M, found by k_qhist / k_qselect below
+            long long k = (long long)P.filter_c * P.n;
+            P.in->q_rank = k < P.M ? k : P.M - 1;
+            P.in->q_prefix = 0;
+            P.in->nlev = 0;                   // level 0 open: n sets, all roots
+            P.in->lv_base = 0;
+            P.in->lv_size = P.n;
+            P.in->lv_roots = P.n;
+            P.in->lv_next = P.n;
         }
+        if (P.threshold_mode == 2)
+            for (int i = tid; i < kQBins; i += blockDim.x) P.qhist[i] = 0;
     }
     if (err) atomicExch(&P.st->status, ECL_MST_ERR_INPUT);
+}
+
+// ---------------------------------------------------------------------------
+// Exact-quantile threshold (threshold_mode 2): the weight
+// of rank c|V| among all M CSR entries -- the target P:143's 20 samples
+// estimate -- by a radix select over the order key u = w ^ 0x80000000 (signed
+// order as unsigned): pass 1 histograms the top 11 bits of every entry, pass
+// 2 the next 11 bits of the entries under the chosen 11-bit prefix, pass 3
+// the last 10 bits under the chosen 22-bit prefix.  k_qselect<PASS> turns a
+// histogram into the next prefix and the rank left below it.
+// ---------------------------------------------------------------------------
+template <int PASS>
+__device__ __forceinline__ void q_bits(int& shift, unsigned& mask) {
+    shift = PASS == 1 ? 21 : PASS == 2 ? 10 : 0;
+    mask = PASS == 3 ? 0x3FFu : 0x7FFu;
+}
+
+template <int PASS>
+__global__ void __launch_bounds__(256) k_qhist(Params P) {
+    __shared__ unsigned h[kQBins];
+    if (!input_ok(P) || __ldg(&P.st->filtered) == 0) return;
+    for (int i = threadIdx.x; i < kQBins; i += blockDim.x) h[i] = 0;
+    __syncthreads();
+    int shift;
+    unsigned mask;
+    q_bits<PASS>(shift, mask);
+    const unsigned prefix = __ldg(&P.in->q_prefix);   // bits above this pass's digit
+    auto add = [&](int w) {
+        const unsigned u = (unsigned)w ^ 0x80000000u;
+        if (PASS == 1 || (u >> (shift + (PASS == 2 ? 11 : 10))) == prefix) atomicAdd(&h[(u >> shift) & mask], 1u);
+    };
+    const long long nq = P.M / 4;
+    const long long stride = (long long)gridDim.x * blockDim.x;
+    for (long long i = (long long)blockIdx.x * blockDim.x + threadIdx.x; i < nq; i += stride) {
+        const int4 w4 = __ldcs(reinterpret_cast<const int4*>(P.eweight) + i);
+        add(w4.x);
+        add(w4.y);
+        add(w4.z);
+        add(w4.w);
+    }
+    for (long long j = nq * 4 + (long long)blockIdx.x * blockDim.x + threadIdx.x; j < P.M; j += stride) add(P.eweight[j]);
+    __syncthreads();
+    for (int i = threadIdx.x; i < kQBins; i += blockDim.x)
+        if (h[i]) atomicAdd(P.qhist + i, (unsigned long long)h[i]);
+}
+
+template <int PASS>
+__global__ void __launch_bounds__(1024) k_qselect(Params P) {
+    __shared__ unsigned long long s_c[kQBins];
+    __shared__ int s_bin;
+    __shared__ long long s_below;
+    if (!input_ok(P) || __ldcg(&P.st->filtered) == 0) return;
+    const int tid = threadIdx.x;
+    for (int i = tid; i < kQBins; i += blockDim.x) {
+        s_c[i] = __ldcg(P.qhist + i);
+        P.qhist[i] = 0;                       // ready for the next pass
+    }
+    __syncthreads();
+    if (tid == 0) {   // 2048 bins: a serial scan is a few microseconds
+        const long long r = __ldcg(&P.in->q_rank);
+        long long cum = 0;
+        int b = 0;
+        for (; b < kQBins - 1; ++b) {
+            if (cum + (long long)s_c[b] > r) break;
+            cum += (long long)s_c[b];
+        }
+        s_bin = b;
+        s_below = cum;
+    }
+    __syncthreads();
+    if (tid == 0) {
+        const int bits = PASS == 3 ? 10 : 11;
+        const unsigned prefix = (__ldcg(&P.in->q_prefix) << bits) | (unsigned)s_bin;
+        P.in->q_prefix = prefix;
+        P.in->q_rank = __ldcg(&P.in->q_rank) - s_below;
+        if (PASS == 3) P.st->threshold = (int)(prefix ^ 0x80000000u);   // phase 1: w < T
+    }
 }
 
 // ---------------------------------------------------------------------------
@@ -114,6 +203,8 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
     const int T = __ldg(&P.st->threshold);
     const bool guard = (P.guards > 0) || (P.guards < 0 && PH == 2);
     const DS D = ds_of(P);
+    // phase 2: set(x) is setid[x] after k_flatten (else a find from parent[x])
+    const int* const sid = P.flatten ? P.setid : P.parent;
     // warp w takes chunks w, w + W, ... (an even sample of the whole CSR, so
     // every region -- and every k_rounds CTA -- gets the same mix even where
     // the density of u < v entries drifts along the rows) and appends its
@@ -311,8 +402,8 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
                     ((__ldg(P.giant_bits + (row[k] >> 5)) >> (row[k] & 31)) & 1)) {
                     pk[k] = qk[k] = giant;                    // both ends in the largest set: filtered
                 } else if (cand[k]) {
-                    pk[k] = (k > 0 && cand[k - 1] && row[k] == row[k - 1]) ? -1 : __ldca(D.par(row[k]));
-                    qk[k] = __ldca(D.par(vv[k]));
+                    pk[k] = (k > 0 && cand[k - 1] && row[k] == row[k - 1]) ? -1 : __ldca(sid + row[k]);
+                    qk[k] = __ldca(sid + vv[k]);
                 }
             }
 #pragma unroll

@@ -10,46 +10,46 @@
 namespace eclmst {
 
 // ---------------------------------------------------------------------------
-// k_flatten: parent[v] = find(v) before the phase-2 populate, so the phase-2
-// populate can use parent[x] as set(x) with one load.  Two launches: stage 1
-// compresses with path halving from every vertex (fast, but a halving store
-// of one thread can land after another thread's final root store and leave
-// a vertex one or two hops from its root); stage 2 finishes exactly with
-// owner-only pointer jumping (each slot written by the thread that owns it,
-// reads through L2 to see the others' progress), cheap on the short paths
-// stage 1 leaves.  Roots never change here.
+// k_flatten: set(v) for every vertex before the phase-2 populate, so
+// that populate reads each endpoint's set with one load.
+//   stage 1: setid[v] = the root of v's set, walking the closed contraction
+//            levels (opts.relabel; each level's root stores its label in the
+//            next one) and then the open level.  The walks halve the paths
+//            they take; with no closed level they also point v at its root
+//            (compression for the phase-2 rounds' finds).  Roots never change
+//            here, so every walk ends at v's root whatever the other threads'
+//            halving stores do.
+//   stage 2: the largest set's membership bitmap (P.giant_bits) from setid.
 // ---------------------------------------------------------------------------
 template <int STAGE>
 __global__ void __launch_bounds__(256) k_flatten(Params P) {
     if (!phase2_needed(P) || !P.flatten) return;
+    if (STAGE == 2 && !P.giant_bits) return;
     const long long stride = (long long)gridDim.x * blockDim.x;
-    const DS D = ds_of(P);
     const int lane = threadIdx.x & 31;
-    const int giant = (STAGE == 2 && P.giant_bits) ? __ldcg(&P.in->giant) : -1;
+    const int nlev = __ldcg(&P.in->nlev);
+    const DS D = ds_of(P);
+    const int giant = STAGE == 2 ? __ldcg(&P.in->giant) : -1;
     // warps walk 32 consecutive vertices together (stage 2 ballots the bitmap)
     for (long long base = (long long)blockIdx.x * blockDim.x + threadIdx.x - lane; base < P.n; base += stride) {
         const long long v = base + lane;
         const bool valid = v < P.n;
         if (STAGE == 1) {
-            // fast, racy compression: path halving by everybody (ends close
-            // to, but not always exactly at, one hop)
             if (valid) {
-                const int r = find_root(D, (int)v, true);
-                if (r != (int)v) *D.par(v) = r;
+                int x = (int)v;
+                for (int l = 0; l < nlev; ++l) {   // closed levels: root -> label in the next level
+                    const int lab = find_label_from(P.parent, x, __ldca(P.parent + x), true);
+                    if (l == 0) P.parent[v] = ~lab;   // v now names its label directly
+                    x = lab;
+                }
+                const int r = find_root(D, x, true);
+                if (nlev == 0 && r != x) *D.par(x) = r;
+                __stcg(P.setid + v, r);
             }
         } else {
-            // exact: owner-only pointer jumping over the now-short paths
-            int p = valid ? __ldcg(D.par(v)) : -1;
-            while (valid) {
-                const int pp = __ldcg(D.par(p));
-                if (pp == p) break;
-                __stcg(D.par(v), pp);
-                p = pp;
-            }
-            if (P.giant_bits) {
-                const unsigned bits = __ballot_sync(kFull, valid && p == giant);
-                if (lane == 0) P.giant_bits[base >> 5] = bits;
-            }
+            const int sv = valid ? __ldcg(P.setid + v) : -1;
+            const unsigned bits = __ballot_sync(kFull, valid && sv == giant);
+            if (lane == 0) P.giant_bits[base >> 5] = bits;
         }
     }
 }
@@ -66,10 +66,9 @@ __global__ void __launch_bounds__(256) k_giant(Params P) {
     __shared__ int s_r[kS];
     __shared__ int s_c[kS];
     if (!phase2_needed(P) || !P.flatten) return;
-    const DS D = ds_of(P);
     const int i = threadIdx.x;
     const long long v = (long long)(splitmix64(0x6A09E667F3BCC909ull + (unsigned long long)i) % (unsigned long long)P.n);
-    s_r[i] = find_root(D, (int)v, false);
+    s_r[i] = __ldcg(P.setid + v);   // k_flatten<1> ran
     __syncthreads();
     // the mode of the samples, exactly (a majority vote misses a set holding
     // less than half of them, e.g. RMAT's giant among many isolated vertices)
@@ -188,13 +187,17 @@ __device__ __forceinline__ RegionSrc region_src(const Params& P, int b, int* s_p
 // split threshold T < INT_MAX (a crowded round, see split_threshold) only the
 // tuples with w < T record their key and go to the front of `out`; the others
 // are deferred to the back of the arena (ending at out_end, count in *s_def).
-template <bool SPLIT = false, class SRC>
-__device__ __forceinline__ void passA(const Params& P, const SRC& S, int4* __restrict__ out, int* s_out,
-                                      bool guard, int T = INT_MAX, int4* out_end = nullptr,
+//
+// MAP: a relabel opened a new contraction
+// level right before this pass, so the tuples still hold ids of the level
+// below, now closed: find() ends at the root's label, its id in the new level
+// (where nothing has hooked yet).  The tuples leave with the new level's ids.
+template <bool SPLIT = false, bool MAP = false, class SRC>
+__device__ __forceinline__ void passA(const Params& P, const DS& D, const SRC& S, int4* __restrict__ out,
+                                      int* s_out, bool guard, int T = INT_MAX, int4* out_end = nullptr,
                                       int* s_def = nullptr) {
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const bool halving = P.halving != 0;
-    const DS D = ds_of(P);
     for (int k = warp; k < S.nloc; k += kWarps) {
         int count;
         const int4* __restrict__ in = S.get(P, k, count);
@@ -217,8 +220,10 @@ __device__ __forceinline__ void passA(const Params& P, const SRC& S, int4* __res
 #pragma unroll
         for (int i = 0; i < kItems; ++i) {
             if (keep[i]) {
-                const int p = find_from(D, t[i].x, px[i], halving);        // L15
-                const int q = find_from(D, t[i].y, qx[i], halving);        // L16
+                const int p = MAP ? find_label_from(D.parent, t[i].x, px[i], halving)   // L15
+                                  : find_from(D, t[i].x, px[i], halving);
+                const int q = MAP ? find_label_from(D.parent, t[i].y, qx[i], halving)   // L16
+                                  : find_from(D, t[i].y, qx[i], halving);
                 keep[i] = p != q;                                          // L17
                 t[i].x = p;                                                // L18: implicit
                 t[i].y = q;                                                //      path compression
@@ -253,9 +258,8 @@ template <class SRC>
 // The MSF weight and edge count go to this warp's shared accumulators once per
 // chunk (acc[0] += weights, acc[1] += edges): no 64-bit running sums held in
 // registers across the loop (k_rounds is register-capped; they spilled).
-__device__ __forceinline__ void passB(const Params& P, const SRC& S, long long* acc) {
+__device__ __forceinline__ void passB(const Params& P, const DS& D, const SRC& S, long long* acc) {
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const DS D = ds_of(P);
     for (int kk = warp; kk < S.nloc; kk += kWarps) {
         // (ECL_B_REVERSE: walk the chunks back to front, so pass B starts on the
         // tuples the last pass wrote most recently, still in L2, and the next
@@ -320,9 +324,9 @@ __device__ __forceinline__ void passB(const Params& P, const SRC& S, long long* 
 // is far larger than L2 (n >= 2^25: every unguarded atomic on a random slot
 // is a DRAM read-modify-write, a guard miss only a read).  Measured: C5 and
 // C4 gain, C2/C3 lose with guards in every round.
-__device__ __forceinline__ bool use_guard(const Params& P, long long live, long long winners) {
+__device__ __forceinline__ bool use_guard(const Params& P, long long live, long long winners, long long slots) {
     if (P.guards >= 0) return P.guards != 0;
-    return live > 8 * winners || P.n >= (1 << 25);
+    return live > 8 * winners || slots >= (1 << 25);
 }
 
 // ---------------------------------------------------------------------------
@@ -394,6 +398,80 @@ __device__ __forceinline__ int split_threshold(const Params& P, const CompactSrc
     return T;
 }
 
+// ---------------------------------------------------------------------------
+// Contraction (opts.relabel).  After pass B the surviving sets of
+// a round are the roots of the open level.  When they are few, they get dense
+// ids 0..R'-1 in a new level: each root r of the old level stores ~label(r)
+// (the level closes), the new level's parent array starts as the identity,
+// and from the next pass A on (which maps the tuples' ids, see passA MAP) the
+// rounds' random accesses -- finds, best-edge slots, hooks -- hit arrays of
+// R' entries instead of n, which stay in L2 once R' is a few million.  The
+// partition, hence every decision of the algorithm, is unchanged: only the
+// names of the sets change.
+//
+// The new level takes the next free id range of parent[] / key[]; its slots
+// start as the identity and inf.  Every CTA
+// scans a contiguous slice of the old level twice -- count the roots, then
+// assign labels in order -- with one grid barrier between the scans and one
+// after.  Returns R' (the same in every CTA).
+// ---------------------------------------------------------------------------
+#ifndef ECL_RELABEL_MIN
+#define ECL_RELABEL_MIN (1 << 21)   // auto: only levels of >= 2M ids (>= 24 MB of key + parent)
+#endif
+__device__ __forceinline__ long long relabel(const Params& P, long long base, long long size, long long nbase,
+                                             cg::grid_group& grid, int* s_wc, long long (*s_red)[kWarps]) {
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int G = gridDim.x, b = blockIdx.x;
+    const long long lo = base + size * b / G, hi = base + size * (b + 1) / G;
+    const long long per = (hi - lo + kWarps - 1) / kWarps;
+    const long long wlo = min(hi, lo + warp * per), whi = min(hi, wlo + per);
+    int c = 0;
+    for (long long x = wlo + lane; x < whi; x += 32) c += __ldcg(P.parent + x) == (int)x;
+    c = warp_sum(c);
+    if (lane == 0) s_wc[warp] = c;
+    __syncthreads();
+    if (tid == 0) {
+        int t = 0;
+        for (int w = 0; w < kWarps; ++w) t += s_wc[w];
+        P.lvcnt[b] = t;
+    }
+    grid.sync();
+    long long before = 0, total = 0;
+    for (int k = tid; k < G; k += kBlock) {
+        const long long v = __ldcg(P.lvcnt + k);
+        total += v;
+        if (k < b) before += v;
+    }
+    before = warp_sum(before);
+    total = warp_sum(total);
+    if (lane == 0) {
+        s_red[0][warp] = before;
+        s_red[1][warp] = total;
+    }
+    __syncthreads();
+    long long at = nbase, tot = 0;
+    for (int w = 0; w < kWarps; ++w) {
+        at += s_red[0][w];
+        tot += s_red[1][w];
+    }
+    for (int w = 0; w < warp; ++w) at += s_wc[w];
+    const unsigned lt = (1u << lane) - 1u;
+    for (long long x0 = wlo; x0 < whi; x0 += 32) {
+        const long long x = x0 + lane;
+        const bool root = x < whi && __ldcg(P.parent + x) == (int)x;
+        const unsigned m = __ballot_sync(kFull, root);
+        if (root) {
+            const int l = (int)(at + __popc(m & lt));
+            __stcg(P.parent + x, ~l);
+            __stcg(P.parent + l, l);
+            __stcg(P.key + l, kInf);
+        }
+        at += __popc(m);
+    }
+    grid.sync();
+    return tot;
+}
+
 template <int PH>
 __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
     cg::grid_group grid = cg::this_grid();
@@ -433,10 +511,25 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
     // arena in buffer hb (-1: none pending), hcnt of them (per CTA; hb is the
     // same in every CTA because every split decision is)
     int hb = -1, hcnt = 0;
+    // the open contraction level (opts.relabel): first id, ids, roots, next
+    // level's first id -- identical in every CTA, touched once per round
+    // only, so kept in shared memory rather than in (capped) registers
+    __shared__ int s_wc[kWarps];
+    __shared__ long long s_lv[4];
+    __shared__ int s_lev;
+    const DS D = ds_of(P);
+    if (tid == 0) {
+        s_lev = __ldcg(&P.in->nlev);
+        s_lv[0] = __ldcg(&P.in->lv_base);
+        s_lv[1] = __ldcg(&P.in->lv_size);
+        s_lv[2] = __ldcg(&P.in->lv_roots);
+        s_lv[3] = __ldcg(&P.in->lv_next);
+    }
+    __syncthreads();
     // one round: pass B over S, then pass A from S into the other worklist
     auto round = [&](const auto& S) {
         const long long w0 = acc[1];
-        passB(P, S, acc);
+        passB(P, D, S, acc);
         const long long d = acc[1] - w0;
         if (lane == 0 && d) atomicAdd(reinterpret_cast<unsigned long long*>(&st->winners[g]), (unsigned long long)d);
         if (tid == 0) s_out = s_def = 0;
@@ -448,22 +541,46 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
             return false;
         }
         const long long win = __ldcg(&st->winners[g]);
-        const bool guard = use_guard(P, L, win);
         ++g;
+        // every winner hooked exactly one root of the open level
+        const long long lv_size = s_lv[1], lv_roots = s_lv[2] - win;
+        // contraction: never while deferred tuples (which keep this level's
+        // ids) wait for their drain
+        bool mapped = false;
+        if (P.relabel != 0 && hb < 0 && s_lev + 1 < kMaxLevels && L > 0 && 2 * lv_roots <= lv_size &&
+            s_lv[3] + lv_roots <= 2LL * P.n &&
+            (P.relabel > 0 || (lv_size >= ECL_RELABEL_MIN && 4 * L >= lv_size))) {
+            const long long nb = s_lv[3];
+            const long long tot = relabel(P, s_lv[0], lv_size, nb, grid, s_wc, s_red);
+            mapped = true;
+            __syncthreads();
+            if (tid == 0) {
+                ++s_lev;
+                s_lv[0] = nb;
+                s_lv[1] = s_lv[2] = tot;
+                s_lv[3] = nb + tot;
+            }
+        } else {
+            __syncthreads();
+            if (tid == 0) s_lv[2] = lv_roots;
+        }
+        __syncthreads();
+        const bool guard = use_guard(P, L, win, s_lv[1]);
         // a split defers to the back of the output arena; with tuples already
         // deferred (hb >= 0) only when that is the same buffer, below them --
         // the deferred set is then one run, drained together (any union of
         // deferred parts is heavier than the light part still running)
         int T = INT_MAX;
         if constexpr (std::is_same<std::decay_t<decltype(S)>, CompactSrc>::value) {
-            if ((hb < 0 || hb == (cur ^ 1)) && crowded(P, L, win, g)) {
+            if (!mapped && (hb < 0 || hb == (cur ^ 1)) && crowded(P, L, win, g)) {
                 T = split_threshold(P, S, L, win, grid, s_w);
                 if (tid == 0) s_def = hb < 0 ? 0 : hcnt;
                 __syncthreads();
             }
         }
-        if (T != INT_MAX) passA<true>(P, S, wl[cur ^ 1], &s_out, guard, T, wl[cur ^ 1] + P.cap, &s_def);
-        else passA(P, S, wl[cur ^ 1], &s_out, guard);
+        if (T != INT_MAX) passA<true>(P, D, S, wl[cur ^ 1], &s_out, guard, T, wl[cur ^ 1] + P.cap, &s_def);
+        else if (mapped) passA<false, true>(P, D, S, wl[cur ^ 1], &s_out, guard);
+        else passA(P, D, S, wl[cur ^ 1], &s_out, guard);
         cur ^= 1;
         __syncthreads();
         C = compact_src(wl[cur], s_out);
@@ -494,7 +611,7 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
         ++g;
         if (tid == 0) s_out = 0;
         __syncthreads();
-        passA(P, H, wl[ob], &s_out, true);
+        passA(P, D, H, wl[ob], &s_out, true);
         cur = ob;
         __syncthreads();
         C = compact_src(wl[cur], s_out);
@@ -523,6 +640,12 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
     }
     if (b0 && tid == 0) {
         P.in->g_end = g;
+        P.in->nlev = s_lev;
+        P.in->lv_base = s_lv[0];
+        P.in->lv_size = s_lv[1];
+        P.in->lv_roots = s_lv[2];
+        P.in->lv_next = s_lv[3];
+        st->relabels = s_lev;
         st->rounds = g + 1;
         st->refilters = __ldcg(&P.in->splits);
         if (overflow) atomicExch(&st->status, ECL_MST_ERR_ROUNDS);

@@ -72,6 +72,7 @@ def test_tiny_adversarial(eclmst, seed):
     g = G.random_small(2 + seed % 9, 3 + (seed * 7) % 40, seed=seed, weights=kinds[seed % 5],
                        multi=seed % 3 == 0, self_loops=seed % 4 == 0)
     assert_parity(eclmst, g)
+    assert_parity(eclmst, g, relabel=1, refilter=seed % 2, filter=seed % 3 - 1)
 
 
 @pytest.mark.parametrize("weights", ["ties", "two", "full", "uniform", "equal"])
@@ -80,6 +81,10 @@ def test_random_multi_tile(eclmst, weights, n, m):
     g = G.random_small(n, m, seed=n + m, weights=weights, multi=True, self_loops=True)
     stats = assert_parity(eclmst, g)
     check_round_bound(g, stats)
+    stats = assert_parity(eclmst, g, relabel=1)
+    check_round_bound(g, stats)
+    if m > n:
+        assert stats["relabels"] >= 1
 
 
 @pytest.mark.parametrize("name", list(synth.CONFIGS))
@@ -104,6 +109,12 @@ def test_config_small(eclmst, name):
     dict(giant_bitmap=1), dict(giant_bitmap=0), dict(giant_bitmap=1, refilter=1),
     dict(giant_bitmap=1, filter=1, threshold_mode=1, threshold=0), dict(giant_bitmap=1, max_ctas=3),
     dict(giant_bitmap=1, atomic_guards=0), dict(giant_bitmap=1, flatten=0),
+    # exact-quantile threshold (NEXT-3)
+    dict(threshold_mode=2), dict(threshold_mode=2, filter=1, filter_c=1), dict(threshold_mode=2, filter_c=64),
+    # contraction to dense set ids (auto only for levels of >= 2M sets): forced at every halving
+    dict(relabel=1), dict(relabel=0), dict(relabel=1, refilter=1), dict(relabel=1, giant_bitmap=1),
+    dict(relabel=1, max_ctas=3), dict(relabel=1, path_halving=0), dict(relabel=1, filter=0),
+    dict(relabel=1, refilter=1, filter=1, filter_c=1, giant_bitmap=1), dict(relabel=1, atomic_guards=1),
 ])
 @pytest.mark.parametrize("name", ["rmat", "uniform", "road"])
 def test_knobs_give_identical_msf(eclmst, name, opts):
@@ -143,13 +154,15 @@ def test_two_valued_weights_nontrivial_phase1(eclmst):
         assert_parity(eclmst, g, filter=1, threshold_mode=1, threshold=1)
 
 
-def test_special_graphs(eclmst):
-    assert_parity(eclmst, G.star_graph(1_000_001, seed=1))                # one 1M-degree row
-    assert_parity(eclmst, G.path_graph(200_000))                         # monotone: deep chain
-    assert_parity(eclmst, G.path_graph(200_000, weights=-torch.arange(199_999)))
-    assert_parity(eclmst, G.complete_graph(700, seed=2, weights="ties"))
-    assert_parity(eclmst, G.cycle_graph(99_999, seed=3, weights="ties"))
-    assert_parity(eclmst, asymmetric_graph())
+@pytest.mark.parametrize("relabel", [-1, 1])
+def test_special_graphs(eclmst, relabel):
+    kw = dict(relabel=relabel)
+    assert_parity(eclmst, G.star_graph(1_000_001, seed=1), **kw)         # one 1M-degree row
+    assert_parity(eclmst, G.path_graph(200_000), **kw)                  # monotone: deep chain
+    assert_parity(eclmst, G.path_graph(200_000, weights=-torch.arange(199_999)), **kw)
+    assert_parity(eclmst, G.complete_graph(700, seed=2, weights="ties"), **kw)
+    assert_parity(eclmst, G.cycle_graph(99_999, seed=3, weights="ties"), **kw)
+    assert_parity(eclmst, asymmetric_graph(), **kw)
     # exactly M = 4n: the filter boundary
     n = 50_000
     a = torch.arange(n, dtype=torch.int64)
@@ -158,7 +171,7 @@ def test_special_graphs(eclmst):
     w = synth.rng.uniform_int31(4, 1, torch.arange(2 * n))
     g = G.csr_from_undirected(n, u, v, w)
     assert g.M == 4 * n
-    st = assert_parity(eclmst, g)
+    st = assert_parity(eclmst, g, **kw)
     assert st["filtered"]
 
 
@@ -266,6 +279,27 @@ def test_host_api_memcpy_variant(eclmst):
         eclmst.ecl_mst(g.n, g.nindex, bad, g.eweight, out)
 
 
+@pytest.mark.parametrize("weights", ["uniform", "full", "ties", "equal", "two"])
+@pytest.mark.parametrize("c", [1, 3, 4, 1000])
+def test_exact_quantile_threshold(eclmst, weights, c):
+    """threshold_mode 2 puts T at the entry of rank min(c n, M - 1) of all M
+    weights (numpy's partition decides the rank independently); the MSF is
+    the oracle's whatever T is."""
+    g = G.random_small(3000 + c, 50_000, seed=c, weights=weights, multi=True, self_loops=True)
+    st = assert_parity(eclmst, g, threshold_mode=2, filter=1, filter_c=c)
+    w = g.eweight.numpy()
+    k = min(c * g.n, g.M - 1)
+    assert st["threshold"] == int(np.partition(w, k)[k])
+    assert st["heavy_edges"] == int(np.count_nonzero(w[oracle_canonical(g)] >= st["threshold"]))
+
+
+def oracle_canonical(g):
+    """Boolean mask of the canonical (u < v) CSR entries."""
+    idx = g.nindex.numpy()
+    rows = np.repeat(np.arange(g.n), np.diff(idx))
+    return rows < g.nlist.numpy()
+
+
 @pytest.mark.parametrize("seed", range(12))
 def test_giant_bitmap_forced_adversarial(eclmst, seed):
     """The n >= 2^25 phase-2 filter (largest-set bitmap) at small n: tie-heavy
@@ -275,7 +309,8 @@ def test_giant_bitmap_forced_adversarial(eclmst, seed):
     n = 500 + 331 * seed
     g = G.random_small(n, 12 * n, seed=4000 + seed, weights=kinds[seed % 6], multi=True, self_loops=True)
     for opts in (dict(giant_bitmap=1), dict(giant_bitmap=1, filter=1, filter_c=2),
-                 dict(giant_bitmap=1, refilter=1, threshold_samples=20, seed=seed)):
+                 dict(giant_bitmap=1, refilter=1, threshold_samples=20, seed=seed),
+                 dict(giant_bitmap=1, relabel=1, refilter=seed % 2)):
         assert_parity(eclmst, g, **opts)
 
 

@@ -17,8 +17,8 @@ for STEP in "$@"; do
            echo "tests rc=$?"; tail -3 gpurun_out/${TAG}_pytest.txt;;
     slow) timeout 3000 python -m pytest tests -q -x -m "gpu and slow" --durations=10 > gpurun_out/${TAG}_pytest_slow.txt 2>&1
           echo "slow rc=$?"; tail -15 gpurun_out/${TAG}_pytest_slow.txt;;
-    bench:*) /usr/bin/time -v timeout 1700 python bench.py --config $CFG > gpurun_out/${TAG}_bench_${CFG}.json 2> gpurun_out/${TAG}_bench_${CFG}.err
-             echo "bench $CFG rc=$?"; grep -E "Maximum resident|Elapsed" gpurun_out/${TAG}_bench_${CFG}.err
+    bench:*) T0=$SECONDS; timeout 1700 python bench.py --config $CFG > gpurun_out/${TAG}_bench_${CFG}.json 2> gpurun_out/${TAG}_bench_${CFG}.err
+             echo "bench $CFG rc=$? wall=$((SECONDS-T0))s"; tail -3 gpurun_out/${TAG}_bench_${CFG}.err
              python tools/bench_brief.py gpurun_out/${TAG}_bench_${CFG}.json;;
     quick:*) timeout 900 python bench.py --config $CFG --parity none --no-e2e --no-cpu-baseline $QUICK_ARGS > gpurun_out/${TAG}_quick_${CFG}.json 2> gpurun_out/${TAG}_quick_${CFG}.err
              echo "quick $CFG rc=$?"; python tools/bench_brief.py gpurun_out/${TAG}_quick_${CFG}.json;;
