@@ -114,6 +114,7 @@ extern "C" {
 
 int ecl_mst_abi_version(void) { return ECL_MST_ABI_VERSION; }
 
+
 const char* ecl_mst_last_error(void) { return g_last_error.c_str(); }
 
 void ecl_mst_default_options(ecl_mst_options* o) {

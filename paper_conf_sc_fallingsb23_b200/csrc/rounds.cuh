@@ -546,23 +546,24 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
         const long long lv_size = s_lv[1], lv_roots = s_lv[2] - win;
         // contraction: never while deferred tuples (which keep this level's
         // ids) wait for their drain
-        bool mapped = false;
-        if (P.relabel != 0 && hb < 0 && s_lev + 1 < kMaxLevels && L > 0 && 2 * lv_roots <= lv_size &&
-            s_lv[3] + lv_roots <= 2LL * P.n &&
-            (P.relabel > 0 || (lv_size >= ECL_RELABEL_MIN && 4 * L >= lv_size))) {
-            const long long nb = s_lv[3];
-            const long long tot = relabel(P, s_lv[0], lv_size, nb, grid, s_wc, s_red);
-            mapped = true;
-            __syncthreads();
-            if (tid == 0) {
+        // (uniform: every input is the same in every thread of every CTA)
+        const bool mapped = P.relabel != 0 && hb < 0 && s_lev + 1 < kMaxLevels && L > 0 &&
+                            2 * lv_roots <= lv_size && s_lv[3] + lv_roots <= 2LL * P.n &&
+                            (P.relabel > 0 || (lv_size >= ECL_RELABEL_MIN && 4 * L >= lv_size));
+        const long long nb = s_lv[3];
+        long long tot = 0;
+        if (mapped) tot = relabel(P, s_lv[0], lv_size, nb, grid, s_wc, s_red);
+        // one barrier, one writer: every thread has read s_lv above
+        __syncthreads();
+        if (tid == 0) {
+            if (mapped) {
                 ++s_lev;
                 s_lv[0] = nb;
                 s_lv[1] = s_lv[2] = tot;
                 s_lv[3] = nb + tot;
+            } else {
+                s_lv[2] = lv_roots;
             }
-        } else {
-            __syncthreads();
-            if (tid == 0) s_lv[2] = lv_roots;
         }
         __syncthreads();
         const bool guard = use_guard(P, L, win, s_lv[1]);

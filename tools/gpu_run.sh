@@ -20,7 +20,7 @@ for STEP in "$@"; do
     bench:*) T0=$SECONDS; timeout 1700 python bench.py --config $CFG > gpurun_out/${TAG}_bench_${CFG}.json 2> gpurun_out/${TAG}_bench_${CFG}.err
              echo "bench $CFG rc=$? wall=$((SECONDS-T0))s"; tail -3 gpurun_out/${TAG}_bench_${CFG}.err
              python tools/bench_brief.py gpurun_out/${TAG}_bench_${CFG}.json;;
-    quick:*) timeout 900 python bench.py --config $CFG --parity none --no-e2e --no-cpu-baseline $QUICK_ARGS > gpurun_out/${TAG}_quick_${CFG}.json 2> gpurun_out/${TAG}_quick_${CFG}.err
+    quick:*) timeout 300 python bench.py --config $CFG --parity none --no-e2e --no-cpu-baseline $QUICK_ARGS > gpurun_out/${TAG}_quick_${CFG}.json 2> gpurun_out/${TAG}_quick_${CFG}.err
              echo "quick $CFG rc=$?"; python tools/bench_brief.py gpurun_out/${TAG}_quick_${CFG}.json;;
     profile:*)
       timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${TAG}_launches_${CFG}.csv \
