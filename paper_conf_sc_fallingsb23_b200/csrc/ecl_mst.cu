@@ -445,6 +445,7 @@ static int run_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t
     // (M >= 4n) the host knows that already and skips the three launches
     const bool maybe_phase2 = P.filter_mode > 0 || (P.filter_mode < 0 && M >= 4LL * n);
     if (e == cudaSuccess && maybe_phase2) {
+        if (P.relabel) k_flatten<0><<<flat_blocks, 256, 0, s>>>(P);
         k_flatten<1><<<flat_blocks, 256, 0, s>>>(P);
         k_giant<<<1, 256, 0, s>>>(P);
         k_flatten<2><<<flat_blocks, 256, 0, s>>>(P);

@@ -12,23 +12,36 @@ namespace eclmst {
 // ---------------------------------------------------------------------------
 // k_flatten: set(v) for every vertex before the phase-2 populate, so
 // that populate reads each endpoint's set with one load.
-//   stage 1: setid[v] = the root of v's set, walking the closed contraction
-//            levels (opts.relabel; each level's root stores its label in the
-//            next one) and then the open level.  The walks halve the paths
-//            they take; with no closed level they also point v at its root
-//            (compression for the phase-2 rounds' finds).  Roots never change
-//            here, so every walk ends at v's root whatever the other threads'
-//            halving stores do.
+//   stage 0: with two or more closed contraction levels (opts.relabel), the
+//            final set of every id of the closed levels above the vertices,
+//            kept in that id's (dead) best-edge slot: each walk climbs the
+//            small upper levels once instead of once per vertex.
+//   stage 1: setid[v] = the root of v's set: a walk in the vertices' level,
+//            then its label's final set (stage 0, or a find in the open level
+//            when it is the only one above).  With no closed level it also
+//            points v at its root (compression for the phase-2 rounds' finds).
+//            Roots never change here, so every walk ends at v's root whatever
+//            the other threads' halving stores do.
 //   stage 2: the largest set's membership bitmap (P.giant_bits) from setid.
 // ---------------------------------------------------------------------------
 template <int STAGE>
 __global__ void __launch_bounds__(256) k_flatten(Params P) {
     if (!phase2_needed(P) || !P.flatten) return;
     if (STAGE == 2 && !P.giant_bits) return;
+    const int nlev = __ldcg(&P.in->nlev);
+    if (STAGE == 0 && nlev < 2) return;
     const long long stride = (long long)gridDim.x * blockDim.x;
     const int lane = threadIdx.x & 31;
-    const int nlev = __ldcg(&P.in->nlev);
     const DS D = ds_of(P);
+    const long long open = __ldcg(&P.in->lv_base);   // first id of the open level
+    if (STAGE == 0) {
+        for (long long x = P.n + (long long)blockIdx.x * blockDim.x + threadIdx.x; x < open; x += stride) {
+            int y = (int)x;
+            while (y < open) y = find_label_from(P.parent, y, __ldca(P.parent + y), true);
+            __stcg(P.key + x, (long long)find_root(D, y, true));
+        }
+        return;
+    }
     const int giant = STAGE == 2 ? __ldcg(&P.in->giant) : -1;
     // warps walk 32 consecutive vertices together (stage 2 ballots the bitmap)
     for (long long base = (long long)blockIdx.x * blockDim.x + threadIdx.x - lane; base < P.n; base += stride) {
@@ -36,14 +49,15 @@ __global__ void __launch_bounds__(256) k_flatten(Params P) {
         const bool valid = v < P.n;
         if (STAGE == 1) {
             if (valid) {
-                int x = (int)v;
-                for (int l = 0; l < nlev; ++l) {   // closed levels: root -> label in the next level
-                    const int lab = find_label_from(P.parent, x, __ldca(P.parent + x), true);
-                    if (l == 0) P.parent[v] = ~lab;   // v now names its label directly
-                    x = lab;
+                int r;
+                if (nlev == 0) {
+                    r = find_root(D, (int)v, true);
+                    if (r != (int)v) *D.par(v) = r;
+                } else {
+                    const int lab = find_label_from(P.parent, (int)v, __ldca(P.parent + v), true);
+                    P.parent[v] = ~lab;   // v now names its label directly
+                    r = nlev == 1 ? find_root(D, lab, true) : (int)__ldcg(P.key + lab);
                 }
-                const int r = find_root(D, x, true);
-                if (nlev == 0 && r != x) *D.par(x) = r;
                 __stcg(P.setid + v, r);
             }
         } else {
@@ -416,17 +430,34 @@ __device__ __forceinline__ int split_threshold(const Params& P, const CompactSrc
 // after.  Returns R' (the same in every CTA).
 // ---------------------------------------------------------------------------
 #ifndef ECL_RELABEL_MIN
-#define ECL_RELABEL_MIN (1 << 21)   // auto: only levels of >= 2M ids (>= 24 MB of key + parent)
+#define ECL_RELABEL_MIN (1 << 21)    // auto: only levels of >= 2M ids (>= 24 MB of key + parent) ...
 #endif
+#ifndef ECL_RELABEL_FIRST
+#define ECL_RELABEL_FIRST (1 << 25)  // ... and the vertices themselves only from 2^25 on (C5): below,
+                                     // parent[] + key[] (12n B) keep enough locality -- measured:
+                                     // C2 2.26 -> 2.37 ms, C3 2.83 -> 3.02 ms, C4 7.31 -> 7.44 ms with it
+#endif
+constexpr int kRlItems = 8;                     // ids per lane per step of a relabel scan
+constexpr int kRlStep = 32 * kRlItems;          // 256 ids per warp step
 __device__ __forceinline__ long long relabel(const Params& P, long long base, long long size, long long nbase,
                                              cg::grid_group& grid, int* s_wc, long long (*s_red)[kWarps]) {
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int G = gridDim.x, b = blockIdx.x;
-    const long long lo = base + size * b / G, hi = base + size * (b + 1) / G;
-    const long long per = (hi - lo + kWarps - 1) / kWarps;
-    const long long wlo = min(hi, lo + warp * per), whi = min(hi, wlo + per);
+    // contiguous steps of 256 ids per warp, in (CTA, warp) order; each lane
+    // keeps 8 independent loads in flight (ids lane, lane + 32, ...)
+    const long long steps = (size + kRlStep - 1) / kRlStep;
+    const long long nw = (long long)G * kWarps, gw = (long long)b * kWarps + warp;
+    const long long s0 = steps * gw / nw, s1 = steps * (gw + 1) / nw;
+    const long long end = base + size;
     int c = 0;
-    for (long long x = wlo + lane; x < whi; x += 32) c += __ldcg(P.parent + x) == (int)x;
+    for (long long st = s0; st < s1; ++st) {
+        const long long x0 = base + st * kRlStep + lane;
+        int v[kRlItems];
+#pragma unroll
+        for (int i = 0; i < kRlItems; ++i) v[i] = x0 + 32 * i < end ? __ldcg(P.parent + x0 + 32 * i) : -1;
+#pragma unroll
+        for (int i = 0; i < kRlItems; ++i) c += v[i] == (int)(x0 + 32 * i);
+    }
     c = warp_sum(c);
     if (lane == 0) s_wc[warp] = c;
     __syncthreads();
@@ -456,17 +487,24 @@ __device__ __forceinline__ long long relabel(const Params& P, long long base, lo
     }
     for (int w = 0; w < warp; ++w) at += s_wc[w];
     const unsigned lt = (1u << lane) - 1u;
-    for (long long x0 = wlo; x0 < whi; x0 += 32) {
-        const long long x = x0 + lane;
-        const bool root = x < whi && __ldcg(P.parent + x) == (int)x;
-        const unsigned m = __ballot_sync(kFull, root);
-        if (root) {
-            const int l = (int)(at + __popc(m & lt));
-            __stcg(P.parent + x, ~l);
-            __stcg(P.parent + l, l);
-            __stcg(P.key + l, kInf);
+    for (long long st = s0; st < s1; ++st) {
+        const long long x0 = base + st * kRlStep + lane;
+        int v[kRlItems];
+#pragma unroll
+        for (int i = 0; i < kRlItems; ++i) v[i] = x0 + 32 * i < end ? __ldcg(P.parent + x0 + 32 * i) : -1;
+#pragma unroll
+        for (int i = 0; i < kRlItems; ++i) {   // labels in id order: item i covers ids x0 + 32 i
+            const long long x = x0 + 32 * i;
+            const bool root = v[i] == (int)x;
+            const unsigned m = __ballot_sync(kFull, root);
+            if (root) {
+                const int l = (int)(at + __popc(m & lt));
+                __stcg(P.parent + x, ~l);
+                __stcg(P.parent + l, l);
+                __stcg(P.key + l, kInf);
+            }
+            at += __popc(m);
         }
-        at += __popc(m);
     }
     grid.sync();
     return tot;
@@ -549,7 +587,8 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
         // (uniform: every input is the same in every thread of every CTA)
         const bool mapped = P.relabel != 0 && hb < 0 && s_lev + 1 < kMaxLevels && L > 0 &&
                             2 * lv_roots <= lv_size && s_lv[3] + lv_roots <= 2LL * P.n &&
-                            (P.relabel > 0 || (lv_size >= ECL_RELABEL_MIN && 4 * L >= lv_size));
+                            (P.relabel > 0 || (lv_size >= ECL_RELABEL_MIN && 4 * L >= lv_size &&
+                                                (s_lev > 0 || lv_size >= ECL_RELABEL_FIRST)));
         const long long nb = s_lv[3];
         long long tot = 0;
         if (mapped) tot = relabel(P, s_lv[0], lv_size, nb, grid, s_wc, s_red);
