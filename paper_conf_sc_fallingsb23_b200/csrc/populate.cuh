@@ -264,12 +264,14 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
         sa = ra <= rl ? __ldg(P.nindex + ra) : LLONG_MAX;
         sz = rz <= rl ? __ldg(P.nindex + rz) : LLONG_MAX;
     };
-    auto vbits = [&](const int (&vv)[kItems]) {
+    // (only entries that can be phase-2 candidates: heavy, and v above the
+    // chunk's first row -- an entry with v <= r0 <= its row is a mirror, L4)
+    auto vbits = [&](const int (&vv)[kItems], const int (&ww)[kItems], int r0) {
         unsigned b = 0;
         if (PH == 2 && giant >= 0) {
 #pragma unroll
             for (int k = 0; k < kItems; ++k)
-                if ((unsigned)vv[k] < (unsigned)P.n)
+                if ((unsigned)vv[k] < (unsigned)P.n && vv[k] > r0 && (!filtered || ww[k] >= T))
                     b |= ((__ldg(P.giant_bits + (vv[k] >> 5)) >> (vv[k] & 31)) & 1u) << k;
         }
         return b;
@@ -292,7 +294,7 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
             starts(nr0, nrl, nsa, nsz);
             if (nxt(lc0) < lend) bracket(nxt(lc0), n2r0, n2rl);
         }
-        nvb = vbits(nv);
+        nvb = vbits(nv, nw, nr0);
     }
     for (long long lc = lc0; lc < lend; lc = nxt(lc)) {
     const long long c = P.shard + lc * P.nshards;
@@ -445,7 +447,7 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
         for (int k = 0; k < kItems; ++k)
             if (keep[k]) rec(t[k].y, make_key(t[k].z, (unsigned)t[k].w));
     }
-    if (PH == 2 && nxt(lc) < lend) nvb = vbits(nv);   // next chunk's far-end bits
+    if (PH == 2 && nxt(lc) < lend) nvb = vbits(nv, nw, nr0);   // next chunk's far-end bits
     // L7: append the chunk's tuples to the warp's region
     unsigned m[kItems];
     int off[kItems];

@@ -268,10 +268,13 @@ __device__ __forceinline__ void passA(const Params& P, const DS& D, const SRC& S
 #define ECL_B_REVERSE 1   // C2 2.319 -> 2.281 ms, C3 2.86 -> 2.83 ms, C4 -0.2%, C1 +-0
 #endif
 // L27-31 (+ L34-37): check, join, mark over the CTA's worklist.
-template <class SRC>
 // The MSF weight and edge count go to this warp's shared accumulators once per
 // chunk (acc[0] += weights, acc[1] += edges): no 64-bit running sums held in
 // registers across the loop (k_rounds is register-capped; they spilled).
+// NORESET: a relabel is expected right after this pass, which abandons this
+// level's best-edge slots, so the winners leave them as they are (k_rounds
+// refills them should the relabel not happen after all).
+template <bool NORESET = false, class SRC>
 __device__ __forceinline__ void passB(const Params& P, const DS& D, const SRC& S, long long* acc) {
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     for (int kk = warp; kk < S.nloc; kk += kWarps) {
@@ -313,8 +316,8 @@ __device__ __forceinline__ void passB(const Params& P, const DS& D, const SRC& S
                 // a mutual pair keeps the smaller representative as root.
                 if (wp && !(wq && p < q)) __stcg(D.par(p), q);
                 if (wq && !(wp && q < p)) __stcg(D.par(q), p);
-                if (wp) __stcg(D.k(p), kInf);                          // L35
-                if (wq) __stcg(D.k(q), kInf);                          // L36
+                if (!NORESET && wp) __stcg(D.k(p), kInf);              // L35
+                if (!NORESET && wq) __stcg(D.k(q), kInf);              // L36
                 P.in_mst[(unsigned)t[i].w] = 1;                        // L31
                 csum += t[i].z;
                 ccnt += 1;
@@ -340,7 +343,7 @@ __device__ __forceinline__ void passB(const Params& P, const DS& D, const SRC& S
 // C4 gain, C2/C3 lose with guards in every round.
 __device__ __forceinline__ bool use_guard(const Params& P, long long live, long long winners, long long slots) {
     if (P.guards >= 0) return P.guards != 0;
-    return live > 8 * winners || slots >= (1 << 25);
+    return live > 8 * winners || slots > (1 << 24);   // (> 128 MB of slots: beyond the L2)
 }
 
 // ---------------------------------------------------------------------------
@@ -565,9 +568,19 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
     }
     __syncthreads();
     // one round: pass B over S, then pass A from S into the other worklist
+    // every relabel condition that does not depend on this round's winners
+    // (the decision itself follows pass B); see passB NORESET
+    auto may_relabel = [&]() {
+        const long long lv_size = s_lv[1];
+        return P.relabel != 0 && hb < 0 && s_lev + 1 < kMaxLevels && L > 0 &&
+               (P.relabel > 0 || (lv_size >= ECL_RELABEL_MIN && 4 * L >= lv_size &&
+                                  (s_lev > 0 || lv_size >= ECL_RELABEL_FIRST)));
+    };
     auto round = [&](const auto& S) {
         const long long w0 = acc[1];
-        passB(P, D, S, acc);
+        const bool noreset = may_relabel();
+        if (noreset) passB<true>(P, D, S, acc);
+        else passB(P, D, S, acc);
         const long long d = acc[1] - w0;
         if (lane == 0 && d) atomicAdd(reinterpret_cast<unsigned long long*>(&st->winners[g]), (unsigned long long)d);
         if (tid == 0) s_out = s_def = 0;
@@ -585,13 +598,17 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
         // contraction: never while deferred tuples (which keep this level's
         // ids) wait for their drain
         // (uniform: every input is the same in every thread of every CTA)
-        const bool mapped = P.relabel != 0 && hb < 0 && s_lev + 1 < kMaxLevels && L > 0 &&
-                            2 * lv_roots <= lv_size && s_lv[3] + lv_roots <= 2LL * P.n &&
-                            (P.relabel > 0 || (lv_size >= ECL_RELABEL_MIN && 4 * L >= lv_size &&
-                                                (s_lev > 0 || lv_size >= ECL_RELABEL_FIRST)));
+        const bool mapped = noreset && 2 * lv_roots <= lv_size && s_lv[3] + lv_roots <= 2LL * P.n;
         const long long nb = s_lv[3];
         long long tot = 0;
-        if (mapped) tot = relabel(P, s_lv[0], lv_size, nb, grid, s_wc, s_red);
+        if (mapped) {
+            tot = relabel(P, s_lv[0], lv_size, nb, grid, s_wc, s_red);
+        } else if (noreset) {   // the level stays open: restore its slots to inf
+            const long long stride = (long long)gridDim.x * kBlock;
+            for (long long x = s_lv[0] + (long long)blockIdx.x * kBlock + tid; x < s_lv[0] + lv_size; x += stride)
+                __stcg(P.key + x, kInf);
+            grid.sync();
+        }
         // one barrier, one writer: every thread has read s_lv above
         __syncthreads();
         if (tid == 0) {
