@@ -55,9 +55,10 @@ def emit(line):
 import torch  # noqa: E402
 
 PEAKS_FILE = os.path.join(ROOT, "MEASURED_PEAKS.json")
-# k_init, k_populate<1>, k_rounds<1>, k_finalize; with filtering also k_flatten<1>, k_giant,
-# k_flatten<2>, k_populate<2>, k_rounds<2>
-LAUNCHES_UNFILTERED, LAUNCHES_FILTERED = 4, 9
+# k_init, k_populate<1>, k_rounds<1>, k_finalize; with filtering also k_flatten<0> (contraction
+# levels), k_flatten<1>, k_giant, k_flatten<2>, k_populate<2>, k_rounds<2>; threshold_mode 2 adds
+# 3 x (k_qhist, k_qselect)
+LAUNCHES_UNFILTERED, LAUNCHES_FILTERED, LAUNCHES_QUANTILE = 4, 10, 6
 CONFIG_NAMES = {"grid": "C1", "road": "C2", "rgg": "C3", "rmat": "C4", "uniform": "C5"}
 # (graph name, n, M, m) of the full-size configs: pure functions of their seeds
 # (synth/); the GPU arm checks them against the generated graph, the
@@ -543,7 +544,8 @@ def main():
         "config": workload_config(args, world, use_dist, opt_kw, gname, n, M, st["canonical_edges"]),
         "ms_per_graph": ms_max, "ms_per_step_all": per_step, "wall_s": wall,
         "edges_per_s_undirected": st["canonical_edges"] / (ms_max / 1e3),
-        "gpu_launches": args.steps * ((LAUNCHES_FILTERED if st["filtered"] else LAUNCHES_UNFILTERED)
+        "gpu_launches": args.steps * ((LAUNCHES_FILTERED + (LAUNCHES_QUANTILE if opt_kw.get("threshold_mode") == 2
+                                                            else 0) if st["filtered"] else LAUNCHES_UNFILTERED)
                                       if not use_dist else 4 + 4 * st["rounds"]),
         "clocks": clocks,
         "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",

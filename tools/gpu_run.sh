@@ -26,7 +26,7 @@ for STEP in "$@"; do
       timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${TAG}_launches_${CFG}.csv \
         python bench.py --config $CFG --steps 2 --warmup 1 --no-e2e --no-cpu-baseline --parity none > gpurun_out/${TAG}_launches_${CFG}.log 2>&1
       echo "launches rc=$?"
-      case $CFG in road|grid) NK=4;; *) NK=9;; esac
+      case $CFG in road|grid) NK=4;; *) NK=10;; esac
       timeout 1500 ncu --set full --clock-control none --import-source on -k regex:"k_" -s $NK -c $NK \
         -o gpurun_out/${TAG}_prof_${CFG} -f python tools/profile_run.py --config $CFG --runs 2 > gpurun_out/${TAG}_prof_${CFG}.log 2>&1
       echo "full rc=$?"; tail -2 gpurun_out/${TAG}_prof_${CFG}.log;;
