@@ -37,6 +37,9 @@ struct Internal {
     int g_end;                         // last global round of the finished phase
     int giant;                         // root of the largest set after phase 1 (-1: none)
     int splits;                        // crowded-round splits taken so far (all phases)
+    unsigned long long tcount;         // populate_mode 1: tuples appended to the one list
+    unsigned long long tcanon, theavy; // populate_mode 1: canonical / deferred edges seen
+    unsigned long long vc_cnt[3];      // drive 2: tuples of the last pass As (round-robin)
     unsigned q_prefix;                 // exact-quantile threshold: bits of the order key fixed so far
     long long q_rank;                  // ... and the rank still to find below that prefix
     // contraction levels (opts.relabel).  Set ids are absolute indices into
@@ -135,6 +138,9 @@ struct Params {
     int relabel;                      // -1 auto, 0 off, 1 whenever the sets at least halved (opts.relabel)
     int* lvcnt;                       // per-CTA root counts of a relabel (kMaxGrid)
     int* setid;                       // set of every vertex after phase 1 (k_flatten), read by populate 2
+    long long wlcap;                  // tuples per worklist buffer (plane stride of opts.tuple_layout 1)
+    int both;                         // opts.both_directions: both directed copies of every edge
+    int drive;                        // opts.drive: 0 data-driven, 1 topology-driven, 2 vertex-centric
     // edge sharding (distributed path; single GPU: shard 0 of 1)
     int shard;                        // global shard id
     int nshards;                      // total shards

@@ -100,10 +100,57 @@ __device__ __forceinline__ void record_min(long long* slot, long long key, bool 
     if (!guard || __ldca(slot) > key) atomicMin(slot, key);
 }
 
+// ---------------------------------------------------------------------------
+// Worklist tuple storage.  The default is the paper's 16-byte 4-tuple
+// <p, q, w, id>, one vector access per tuple.  SOA is the "No
+// Tuples" de-optimisation: the four items in four int planes
+// `stride` tuples apart.  A tuple pointer is the int4* of a range's first
+// tuple (AoS) or the address of that tuple's plane-0 int, cast to int4*
+// (SoA); tadd() moves it by tuples either way.
+// ---------------------------------------------------------------------------
+template <bool SOA>
+__device__ __forceinline__ int4* tadd(int4* p, long long n) {
+    return SOA ? reinterpret_cast<int4*>(reinterpret_cast<int*>(p) + n) : p + n;
+}
+template <bool SOA>
+__device__ __forceinline__ const int4* tadd(const int4* p, long long n) {
+    return SOA ? reinterpret_cast<const int4*>(reinterpret_cast<const int*>(p) + n) : p + n;
+}
+// streaming load (read once), L2 load, L2 store, and the weight alone
+template <bool SOA>
+__device__ __forceinline__ int4 tld_cs(const int4* p, long long i, long long stride) {
+    if (!SOA) return __ldcs(p + i);
+    const int* q = reinterpret_cast<const int*>(p) + i;
+    return make_int4(__ldcs(q), __ldcs(q + stride), __ldcs(q + 2 * stride), __ldcs(q + 3 * stride));
+}
+template <bool SOA>
+__device__ __forceinline__ int4 tld_cg(const int4* p, long long i, long long stride) {
+    if (!SOA) return __ldcg(p + i);
+    const int* q = reinterpret_cast<const int*>(p) + i;
+    return make_int4(__ldcg(q), __ldcg(q + stride), __ldcg(q + 2 * stride), __ldcg(q + 3 * stride));
+}
+template <bool SOA>
+__device__ __forceinline__ void tst_cg(int4* p, long long i, int4 t, long long stride) {
+    if (!SOA) {
+        __stcg(p + i, t);
+        return;
+    }
+    int* q = reinterpret_cast<int*>(p) + i;
+    __stcg(q, t.x);
+    __stcg(q + stride, t.y);
+    __stcg(q + 2 * stride, t.z);
+    __stcg(q + 3 * stride, t.w);
+}
+template <bool SOA>
+__device__ __forceinline__ int tld_w(const int4* p, long long i, long long stride) {
+    return SOA ? __ldcg(reinterpret_cast<const int*>(p) + i + 2 * stride) : __ldcg(&p[i].z);
+}
+
 // Warp-level compaction of one chunk (kItems tuples per lane, any order):
 // one shared-memory atomicAdd per warp reserves the output range.
+template <bool SOA = false>
 __device__ __forceinline__ int warp_emit(const int4 (&t)[kItems], const bool (&keep)[kItems],
-                                         int4* __restrict__ out, int* s_out) {
+                                         int4* __restrict__ out, int* s_out, long long stride = 0) {
     const int lane = threadIdx.x & 31;
     unsigned m[kItems];
     int off[kItems];
@@ -120,14 +167,15 @@ __device__ __forceinline__ int warp_emit(const int4 (&t)[kItems], const bool (&k
     const unsigned lt = (1u << lane) - 1u;
 #pragma unroll
     for (int i = 0; i < kItems; ++i)
-        if (keep[i]) __stcg(out + base + off[i] + __popc(m[i] & lt), t[i]);
+        if (keep[i]) tst_cg<SOA>(out, base + off[i] + __popc(m[i] & lt), t[i], stride);
     return tot;
 }
 
 // Same, for the tuples a crowded-round split defers: they fill the arena from
 // its end downwards ([end - total, end) after the pass, contiguous).
+template <bool SOA = false>
 __device__ __forceinline__ void warp_emit_back(const int4 (&t)[kItems], const bool (&keep)[kItems],
-                                               int4* __restrict__ end, int* s_cnt) {
+                                               int4* __restrict__ end, int* s_cnt, long long stride = 0) {
     const int lane = threadIdx.x & 31;
     unsigned m[kItems];
     int off[kItems];
@@ -142,11 +190,11 @@ __device__ __forceinline__ void warp_emit_back(const int4 (&t)[kItems], const bo
     int base = 0;
     if (lane == 0) base = atomicAdd(s_cnt, tot);
     base = __shfl_sync(kFull, base, 0);
-    int4* dst = end - base - tot;
+    int4* dst = tadd<SOA>(end, -(long long)(base + tot));
     const unsigned lt = (1u << lane) - 1u;
 #pragma unroll
     for (int i = 0; i < kItems; ++i)
-        if (keep[i]) __stcg(dst + off[i] + __popc(m[i] & lt), t[i]);
+        if (keep[i]) tst_cg<SOA>(dst, off[i] + __popc(m[i] & lt), t[i], stride);
 }
 
 // warp-cooperative 32-ary search: largest r in [0, n) with nindex[r] <= x.

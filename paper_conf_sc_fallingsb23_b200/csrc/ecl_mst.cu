@@ -187,6 +187,25 @@ static inline bool giant_bitmap_on(int32_t opt, int32_t n) {
     return opt > 0 || (opt < 0 && (long long)n >= ECL_GIANT_MIN_N);
 }
 
+// the instantiation for the de-optimisation knobs (opts.tuple_layout,
+// both_directions, drive); the defaults pick <PH, false, ...0>
+template <int PH>
+static void (*pop_kernel(bool soa, int both))(Params) {
+    if (soa) return both ? k_populate<PH, true, true> : k_populate<PH, true, false>;
+    return both ? k_populate<PH, false, true> : k_populate<PH, false, false>;
+}
+template <int PH>
+static const void* rounds_kernel(bool soa, int drive) {
+    if (soa) {
+        if (drive == 1) return reinterpret_cast<const void*>(k_rounds<PH, true, 1>);
+        if (drive == 2) return reinterpret_cast<const void*>(k_rounds<PH, true, 2>);
+        return reinterpret_cast<const void*>(k_rounds<PH, true, 0>);
+    }
+    if (drive == 1) return reinterpret_cast<const void*>(k_rounds<PH, false, 1>);
+    if (drive == 2) return reinterpret_cast<const void*>(k_rounds<PH, false, 2>);
+    return reinterpret_cast<const void*>(k_rounds<PH, false, 0>);
+}
+
 // threshold_mode 2: the three radix-select passes after k_init (the kernels
 // return at once when the graph is not filtered)
 static cudaError_t launch_quantile(const Params& P, const DevInfo& di, cudaStream_t s) {
@@ -231,8 +250,9 @@ static int run_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t
     ecl_mst_default_options(&o);
     if (opts) o = *opts;
     if (o.threshold_mode < 0 || o.threshold_mode > 2) return fail(ECL_MST_ERR_INVALID, "threshold_mode must be 0, 1 or 2");
-    if (o.populate_mode || o.both_directions || o.tuple_layout || o.drive)
-        return fail(ECL_MST_ERR_INVALID, "de-optimisation knob not available");
+    if (o.populate_mode < 0 || o.populate_mode > 1 || o.both_directions < 0 || o.both_directions > 1 ||
+        o.tuple_layout < 0 || o.tuple_layout > 1 || o.drive < 0 || o.drive > 2)
+        return fail(ECL_MST_ERR_INVALID, "populate_mode, both_directions, tuple_layout in {0,1}; drive in {0,1,2}");
     const Layout L = layout_for(n, M, o.both_directions ? 2 : 1);
     if (workspace_bytes < L.total) return fail(ECL_MST_ERR_WORKSPACE, "workspace %zu < %zu bytes", workspace_bytes, L.total);
     if (reinterpret_cast<uintptr_t>(workspace) % 256) return fail(ECL_MST_ERR_WORKSPACE, "workspace not 256-byte aligned");
@@ -274,7 +294,8 @@ static int run_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t
         case 3: contig = 1; break;
         default: contig = 1; break;
     }
-    const long long rcap = ceil_div(nchunks, W) * kChunk;
+    // (both_directions: every candidate edge takes two tuples)
+    const long long rcap = ceil_div(nchunks, W) * kChunk * (o.both_directions ? 2 : 1);
     // only warps that own a block write a region
     if (W * rcap > L.wl_cap) return fail(ECL_MST_ERR_WORKSPACE, "internal: regions exceed worklist capacity");
     // k_rounds arenas: the worklist of CTA b never exceeds its first input,
@@ -327,6 +348,15 @@ static int run_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t
     P.relabel = (o.flatten && (long long)n <= (1LL << 30)) ? (o.relabel < 0 ? -1 : (o.relabel ? 1 : 0)) : 0;
     P.lvcnt = reinterpret_cast<int*>(ws + L.lvcnt);
     P.setid = reinterpret_cast<int*>(ws + L.setid);
+    P.wlcap = L.wl_cap;
+    P.both = o.both_directions ? 1 : 0;
+    P.drive = o.drive;
+    if (o.drive) {   // the topology-driven passes re-read the phase's edges: no splits, no contraction
+        P.refilter = 0;
+        P.relabel = 0;
+    }
+    const bool soa = o.tuple_layout == 1;
+    const bool thread_pop = o.populate_mode == 1;
     P.shard = 0;
     P.nshards = 1;
     P.nlocal = nchunks;
@@ -378,7 +408,7 @@ static int run_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t
     };
     const unsigned flat_blocks = (unsigned)std::max<long long>(init_blocks, 1);
     // staged upload: CTA groups of the phase-1 populate and their CSR pieces
-    const bool staged = stg && (contig & 1);
+    const bool staged = stg && (contig & 1) && !thread_pop;
     const int pieces = staged ? (int)std::min<long long>(kStagePieces, pop_blocks) : 1;
     auto group_cta = [&](int k) { return (long long)(pop_blocks * k / pieces); };
     cudaError_t e = cudaSuccess;
@@ -432,14 +462,19 @@ static int run_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t
                     e = cudaGetLastError();
                 }
             }
+        } else if (thread_pop) {   // opts.populate_mode 1
+            if (soa) k_populate_thread<1, true><<<flat_blocks, 256, 0, s>>>(P);
+            else k_populate_thread<1, false><<<flat_blocks, 256, 0, s>>>(P);
+            k_regions<1><<<1, 256, 0, s>>>(P);
+            e = cudaGetLastError();
         } else {
-            k_populate<1><<<(unsigned)pop_blocks, kPopBlock, 0, s>>>(P);
+            pop_kernel<1>(soa, P.both)<<<(unsigned)pop_blocks, kPopBlock, 0, s>>>(P);
             e = cudaGetLastError();
         }
     }
     if (e == cudaSuccess) e = mark();
     if (e == cudaSuccess)
-        e = cudaLaunchCooperativeKernel(reinterpret_cast<const void*>(k_rounds<1>), dim3((unsigned)G), dim3(kBlock), args, 0, s);
+        e = cudaLaunchCooperativeKernel(rounds_kernel<1>(soa, P.drive), dim3((unsigned)G), dim3(kBlock), args, 0, s);
     if (e == cudaSuccess) e = mark();
     // phase 2 can only happen when filtering is on; with the automatic rule
     // (M >= 4n) the host knows that already and skips the three launches
@@ -453,12 +488,18 @@ static int run_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t
     }
     if (e == cudaSuccess) e = mark();
     if (e == cudaSuccess && maybe_phase2) {
-        k_populate<2><<<(unsigned)pop_blocks, kPopBlock, 0, s>>>(P);
+        if (thread_pop) {
+            if (soa) k_populate_thread<2, true><<<flat_blocks, 256, 0, s>>>(P);
+            else k_populate_thread<2, false><<<flat_blocks, 256, 0, s>>>(P);
+            k_regions<2><<<1, 256, 0, s>>>(P);
+        } else {
+            pop_kernel<2>(soa, P.both)<<<(unsigned)pop_blocks, kPopBlock, 0, s>>>(P);
+        }
         e = cudaGetLastError();
     }
     if (e == cudaSuccess) e = mark();
     if (e == cudaSuccess && maybe_phase2)
-        e = cudaLaunchCooperativeKernel(reinterpret_cast<const void*>(k_rounds<2>), dim3((unsigned)G), dim3(kBlock), args, 0, s);
+        e = cudaLaunchCooperativeKernel(rounds_kernel<2>(soa, P.drive), dim3((unsigned)G), dim3(kBlock), args, 0, s);
     if (e == cudaSuccess) e = mark();
     if (e == cudaSuccess) {
         k_finalize<<<1, 32, 0, s>>>(P);
@@ -920,6 +961,9 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
         P.relabel = 0;   // (the replicated union-find stays on vertex ids)
         P.lvcnt = nullptr;
         P.setid = reinterpret_cast<int*>(ws + L.setid);
+        P.wlcap = L.wl_cap;
+        P.both = 0;
+        P.drive = 0;
         P.shard = shard;
         P.nshards = (int)Pt;
         P.nlocal = nlocal;

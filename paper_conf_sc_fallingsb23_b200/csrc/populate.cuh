@@ -76,6 +76,8 @@ __global__ void __launch_bounds__(256) k_init(Params P) {
             P.in->done = 0;
             P.in->giant = -1;
             P.in->splits = 0;
+            P.in->tcount = P.in->tcanon = P.in->theavy = 0;
+            P.in->vc_cnt[0] = P.in->vc_cnt[1] = P.in->vc_cnt[2] = 0;
             // exact quantile (threshold_mode 2): the entry of rank c|V| (0-based,
             // at most M - 1) among all M, found by k_qhist / k_qselect below
             long long k = (long long)P.filter_c * P.n;
@@ -173,7 +175,7 @@ __global__ void __launch_bounds__(1024) k_qselect(Params P) {
 // ---------------------------------------------------------------------------
 // k_populate<PH>: one warp per 128-entry CSR chunk
 // ---------------------------------------------------------------------------
-template <int PH>
+template <int PH, bool SOA = false, bool BOTH = false>
 #ifndef ECL_DEEP_PH1
 #define ECL_DEEP_PH1 0
 #endif
@@ -211,7 +213,7 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
     // tuples densely to its own region: no atomics, no CTA barrier.
     const int w = (P.pop_cta0 + (int)blockIdx.x) * kPopWarps + warp;
     if (w >= P.W) return;   // (sharded path: partial last CTA)
-    int4* const out = P.wl0 + (long long)w * P.rcap;
+    int4* const out = tadd<SOA>(P.wl0, (long long)w * P.rcap);
     int cnt = 0, canon_cnt = 0, heavy_cnt = 0;
     bool err = false;
     const int p0 = lane * kItems;
@@ -446,23 +448,36 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
 #pragma unroll
         for (int k = 0; k < kItems; ++k)
             if (keep[k]) rec(t[k].y, make_key(t[k].z, (unsigned)t[k].w));
+        if (BOTH) {   // opts.both_directions: the mirror copy records the same key again
+#pragma unroll
+            for (int k = 0; k < kItems; ++k) {
+                if (keep[k]) {
+                    rec(t[k].y, make_key(t[k].z, (unsigned)t[k].w));
+                    rec(t[k].x, make_key(t[k].z, (unsigned)t[k].w));
+                }
+            }
+        }
     }
     if (PH == 2 && nxt(lc) < lend) nvb = vbits(nv, nw, nr0);   // next chunk's far-end bits
-    // L7: append the chunk's tuples to the warp's region
-    unsigned m[kItems];
-    int off[kItems];
-    int tot = 0;
+    // L7: append the chunk's tuples to the warp's region (both_directions:
+    // then their mirror copies <q, p, w, id>)
+    for (int copy = 0; copy < 1 + BOTH; ++copy) {
+        unsigned m[kItems];
+        int off[kItems];
+        int tot = 0;
 #pragma unroll
-    for (int i = 0; i < kItems; ++i) {
-        m[i] = __ballot_sync(kFull, keep[i]);
-        off[i] = tot;
-        tot += __popc(m[i]);
+        for (int i = 0; i < kItems; ++i) {
+            m[i] = __ballot_sync(kFull, keep[i]);
+            off[i] = tot;
+            tot += __popc(m[i]);
+            if (copy) t[i] = make_int4(t[i].y, t[i].x, t[i].z, t[i].w);
+        }
+        const unsigned lt = (1u << lane) - 1u;
+#pragma unroll
+        for (int i = 0; i < kItems; ++i)
+            if (keep[i]) tst_cg<SOA>(out, cnt + off[i] + __popc(m[i] & lt), t[i], P.wlcap);
+        cnt += tot;
     }
-    const unsigned lt = (1u << lane) - 1u;
-#pragma unroll
-    for (int i = 0; i < kItems; ++i)
-        if (keep[i]) __stcg(out + cnt + off[i] + __popc(m[i] & lt), t[i]);
-    cnt += tot;
     }
     if (err) atomicExch(&P.st->status, ECL_MST_ERR_INPUT);
     if (PH == 2 && kg >= 0) {
@@ -475,6 +490,95 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
         heavy_cnt = warp_sum(heavy_cnt);
     }
     if (lane == 0) P.region[w] = make_int4(cnt, canon_cnt, heavy_cnt, 0);
+}
+
+// ---------------------------------------------------------------------------
+// opts.populate_mode 1, "Thread-Based": one thread per vertex walks
+// its whole adjacency list -- the loop on Line 3 is never spread over a warp
+// -- and appends each tuple to one list with a global atomicAdd (P:154
+// "Lines 7 and 18"); k_regions then cuts that list into the populate regions
+// k_rounds reads.  Same tuples, keys and counts as k_populate.
+// ---------------------------------------------------------------------------
+template <int PH, bool SOA = false>
+__global__ void __launch_bounds__(256) k_populate_thread(Params P) {
+    if (!input_ok(P)) return;
+    if (PH == 2 && !phase2_needed(P)) return;
+    if (blockIdx.x == 0 && threadIdx.x == 0) P.st->t_ns[PH == 1 ? 1 : 3] = (long long)globaltimer_ns();
+    const bool filtered = __ldg(&P.st->filtered) != 0;
+    const int T = __ldg(&P.st->threshold);
+    const bool guard = (P.guards > 0) || (P.guards < 0 && PH == 2);
+    const bool halving = P.halving != 0;
+    const DS D = ds_of(P);
+    const long long stride = (long long)gridDim.x * blockDim.x;
+    long long canon = 0, heavy = 0;
+    bool err = false;
+    for (long long u = (long long)blockIdx.x * blockDim.x + threadIdx.x; u < P.n; u += stride) {
+        const long long s0 = P.nindex[u], s1 = P.nindex[u + 1];
+        int pu = -1;
+        for (long long j = s0; j < s1; ++j) {                      // L3: this thread, every entry
+            const int v = P.nlist[j], w = P.eweight[j];
+            if (PH == 1 && P.zero_mst) P.in_mst[j] = 0;
+            if ((unsigned)v >= (unsigned)P.n) {
+                err = true;
+                continue;
+            }
+            if (!((int)u < v)) continue;                            // L4
+            const bool hv = filtered && w >= T;                     // L6
+            if (PH == 1) {
+                ++canon;
+                heavy += hv;
+                if (hv) continue;
+            } else if (!hv) {
+                continue;
+            }
+            int p = (int)u, q = v;
+            if (PH == 2) {   // set(u), set(v)
+                if (pu < 0) pu = P.flatten ? __ldca(P.setid + u) : find_root(D, (int)u, halving);
+                p = pu;
+                q = P.flatten ? __ldca(P.setid + v) : find_root(D, v, halving);
+                if (p == q) continue;
+            }
+            const long long key = make_key(w, (unsigned)j);
+            const unsigned long long at = atomicAdd(&P.in->tcount, 1ull + P.both);   // L7
+            tst_cg<SOA>(P.wl0, (long long)at, make_int4(p, q, w, (int)(unsigned)j), P.wlcap);
+            if (P.both) tst_cg<SOA>(P.wl0, (long long)at + 1, make_int4(q, p, w, (int)(unsigned)j), P.wlcap);
+            for (int c = 0; c < 1 + P.both; ++c) {                  // round 0's L20-21
+                record_min(D.k(p), key, guard);
+                record_min(D.k(q), key, guard);
+            }
+        }
+    }
+    if (err) atomicExch(&P.st->status, ECL_MST_ERR_INPUT);
+    if (PH == 1) {
+        canon = warp_sum(canon);
+        heavy = warp_sum(heavy);
+        if ((threadIdx.x & 31) == 0) {
+            if (canon) atomicAdd(&P.in->tcanon, (unsigned long long)canon);
+            if (heavy) atomicAdd(&P.in->theavy, (unsigned long long)heavy);
+        }
+    }
+}
+
+// the one list of k_populate_thread as populate regions: region w holds its
+// tuples [w rcap, (w + 1) rcap), and its share of the phase-1 counts.  Resets
+// the list counter for the next phase.
+template <int PH>
+__global__ void __launch_bounds__(256) k_regions(Params P) {
+    if (!input_ok(P)) return;
+    if (PH == 2 && !phase2_needed(P)) return;
+    const long long K = (long long)__ldcg(&P.in->tcount);
+    const long long canon = PH == 1 ? (long long)__ldcg(&P.in->tcanon) : 0;
+    const long long heavy = PH == 1 ? (long long)__ldcg(&P.in->theavy) : 0;
+    for (int w = threadIdx.x; w < P.W; w += blockDim.x) {
+        const long long c = min(P.rcap, max(0LL, K - (long long)w * P.rcap));
+        // (region counts are int: the host keeps rcap below 2^30, and the
+        // phase-1 totals are spread evenly over the regions)
+        const long long W = P.W;
+        P.region[w] = make_int4((int)c, (int)(canon * (w + 1) / W - canon * w / W),
+                                (int)(heavy * (w + 1) / W - heavy * w / W), 0);
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) P.in->tcount = 0;
 }
 
 }  // namespace eclmst

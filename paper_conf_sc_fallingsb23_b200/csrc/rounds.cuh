@@ -108,17 +108,23 @@ __global__ void __launch_bounds__(256) k_giant(Params P) {
 // search over the shared prefix s_pre) -- RegionSrc; after a pass A it is one
 // compact run of cnt tuples -- CompactSrc.  Two types, so each pass is
 // compiled once per mode and carries only the registers that mode needs.
-struct CompactSrc {
+// (SOA: the tuples are stored as four planes, opts.tuple_layout; see tadd.)
+template <bool SOA_ = false>
+struct CompactSrcT {
+    static constexpr bool SOA = SOA_;
     const int4* base;
     int cnt;
     int nloc;
     __device__ __forceinline__ const int4* get(const Params&, int j, int& count) const {
         count = min(kChunk, cnt - j * kChunk);
-        return base + (long long)j * kChunk;
+        return tadd<SOA>(base, (long long)j * kChunk);
     }
 };
+using CompactSrc = CompactSrcT<false>;
 
-struct RegionSrc {
+template <bool SOA_ = false>
+struct RegionSrcT {
+    static constexpr bool SOA = SOA_;
     const int* s_pre;   // shared memory: chunk prefix per region (nreg + 1)
     const int* s_rcnt;  // shared memory: tuples per region
     int nreg;
@@ -133,12 +139,44 @@ struct RegionSrc {
         }
         const int off = j - s_pre[lo];
         count = min(kChunk, s_rcnt[lo] - off * kChunk);
-        return P.wl0 + (long long)(first_w + lo * P.G) * P.rcap + (long long)off * kChunk;
+        return tadd<SOA>(P.wl0, (long long)(first_w + lo * P.G) * P.rcap + (long long)off * kChunk);
+    }
+};
+using RegionSrc = RegionSrcT<false>;
+
+// pass B's view of the one list a vertex-centric pass A appends to (opts.drive
+// 2): CTA b reads the list's chunks b, b + G, ...
+template <bool SOA_ = false>
+struct GlobalSrcT {
+    static constexpr bool SOA = SOA_;
+    const int4* base;
+    long long cnt;
+    int nloc;
+    __device__ __forceinline__ const int4* get(const Params&, int j, int& count) const {
+        const long long c = blockIdx.x + (long long)j * gridDim.x;
+        count = (int)min((long long)kChunk, cnt - c * kChunk);
+        return tadd<SOA>(base, c * kChunk);
     }
 };
 
-__device__ __forceinline__ CompactSrc compact_src(const int4* base, int cnt) {
-    CompactSrc S;
+template <bool SOA = false>
+__device__ __forceinline__ GlobalSrcT<SOA> global_src(const int4* base, long long cnt) {
+    GlobalSrcT<SOA> S;
+    S.base = base;
+    S.cnt = cnt;
+    const long long nch = (cnt + kChunk - 1) / kChunk;
+    S.nloc = blockIdx.x < nch ? (int)((nch - blockIdx.x + gridDim.x - 1) / gridDim.x) : 0;
+    return S;
+}
+
+template <class T>
+struct is_compact_src : std::false_type {};
+template <bool S2>
+struct is_compact_src<CompactSrcT<S2>> : std::true_type {};
+
+template <bool SOA = false>
+__device__ __forceinline__ CompactSrcT<SOA> compact_src(const int4* base, int cnt) {
+    CompactSrcT<SOA> S;
     S.base = base;
     S.cnt = cnt;
     S.nloc = (cnt + kChunk - 1) / kChunk;
@@ -149,11 +187,12 @@ __device__ __forceinline__ CompactSrc compact_src(const int4* base, int cnt) {
 // counts into shared memory, builds the chunk prefix, and adds the kept,
 // canonical and deferred counts to the stats (phase 1 counters only if
 // count_phase1).  Every thread of the CTA must call it.
-__device__ __forceinline__ RegionSrc region_src(const Params& P, int b, int* s_pre, int* s_rcnt,
-                                                long long (*s_red)[kWarps], int64_t* live_slot,
-                                                bool count_phase1) {
+template <bool SOA = false>
+__device__ __forceinline__ RegionSrcT<SOA> region_src(const Params& P, int b, int* s_pre, int* s_rcnt,
+                                                      long long (*s_red)[kWarps], int64_t* live_slot,
+                                                      bool count_phase1) {
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    RegionSrc R;
+    RegionSrcT<SOA> R;
     R.s_pre = s_pre;
     R.s_rcnt = s_rcnt;
     R.nreg = b < P.W ? (P.W - b + P.G - 1) / P.G : 0;
@@ -221,7 +260,7 @@ __device__ __forceinline__ void passA(const Params& P, const DS& D, const SRC& S
         for (int i = 0; i < kItems; ++i) {
             const int idx = i * 32 + lane;
             keep[i] = idx < count;
-            t[i] = keep[i] ? __ldcs(in + idx) : make_int4(0, 0, 0, 0);
+            t[i] = keep[i] ? tld_cs<SRC::SOA>(in, idx, P.wlcap) : make_int4(0, 0, 0, 0);
         }
         int px[kItems], qx[kItems];
 #pragma unroll
@@ -250,7 +289,7 @@ __device__ __forceinline__ void passA(const Params& P, const DS& D, const SRC& S
                 heavy[i] = keep[i] && t[i].z >= T;
                 keep[i] = keep[i] && t[i].z < T;
             }
-            warp_emit_back(t, heavy, out_end, s_def);
+            warp_emit_back<SRC::SOA>(t, heavy, out_end, s_def, P.wlcap);
         }
 #pragma unroll
         for (int i = 0; i < kItems; ++i) {
@@ -260,7 +299,40 @@ __device__ __forceinline__ void passA(const Params& P, const DS& D, const SRC& S
                 record_min(D.k(t[i].y), key, guard);                      // L21
             }
         }
-        warp_emit(t, keep, out, s_out);                                   // L18
+        warp_emit<SRC::SOA>(t, keep, out, s_out, P.wlcap);                // L18
+    }
+}
+
+// opts.drive 2, "Vertex-Centric": pass A as one thread per vertex
+// walking its CSR row in every round -- topology-driven, all edges of the
+// phase: p = find(u) once per vertex, q = find(v) per edge (no tuple carries
+// representatives between rounds); live edges record their key (L19-21) and
+// are appended to one list (global atomicAdd) that pass B reads.
+template <int PH, bool SOA>
+__device__ __forceinline__ void passA_vc(const Params& P, const DS& D, unsigned long long* cnt, bool guard) {
+    const bool filtered = __ldg(&P.st->filtered) != 0;
+    const int T = __ldg(&P.st->threshold);
+    const bool halving = P.halving != 0;
+    const long long stride = (long long)gridDim.x * kBlock;
+    for (long long u = (long long)blockIdx.x * kBlock + threadIdx.x; u < P.n; u += stride) {
+        const long long s0 = __ldg(P.nindex + u), s1 = __ldg(P.nindex + u + 1);
+        int pu = -1;
+        for (long long j = s0; j < s1; ++j) {
+            const int v = __ldg(P.nlist + j);
+            if ((unsigned)v >= (unsigned)P.n || !((int)u < v)) continue;          // L4
+            const int w = __ldg(P.eweight + j);
+            const bool hv = filtered && w >= T;
+            if (PH == 1 ? hv : !hv) continue;                                     // this phase's edges
+            if (pu < 0) pu = find_root(D, (int)u, halving);                      // L15
+            const int q = find_root(D, v, halving);                              // L16
+            if (pu == q) continue;                                               // L17
+            const long long key = make_key(w, (unsigned)j);                      // L19
+            record_min(D.k(pu), key, guard);                                     // L20
+            record_min(D.k(q), key, guard);                                      // L21
+            const unsigned long long at = atomicAdd(cnt, 1ull + P.both);
+            tst_cg<SOA>(P.wl1, (long long)at, make_int4(pu, q, w, (int)(unsigned)j), P.wlcap);
+            if (P.both) tst_cg<SOA>(P.wl1, (long long)at + 1, make_int4(q, pu, w, (int)(unsigned)j), P.wlcap);
+        }
     }
 }
 
@@ -290,7 +362,7 @@ __device__ __forceinline__ void passB(const Params& P, const DS& D, const SRC& S
         for (int i = 0; i < kItems; ++i) {
             const int idx = i * 32 + lane;
             ok[i] = idx < count;
-            t[i] = ok[i] ? __ldcg(in + idx) : make_int4(0, 0, 0, 0);
+            t[i] = ok[i] ? tld_cg<SRC::SOA>(in, idx, P.wlcap) : make_int4(0, 0, 0, 0);
         }
         // Only the id half of each slot is compared: ids are unique per
         // edge, so id equality is key equality (and inf's id half, 2^32-1,
@@ -319,8 +391,12 @@ __device__ __forceinline__ void passB(const Params& P, const DS& D, const SRC& S
                 if (!NORESET && wp) __stcg(D.k(p), kInf);              // L35
                 if (!NORESET && wq) __stcg(D.k(q), kInf);              // L36
                 P.in_mst[(unsigned)t[i].w] = 1;                        // L31
-                csum += t[i].z;
-                ccnt += 1;
+                // (both_directions: the edge's two copies make the same
+                // hooks and marks; only the p < q copy counts it)
+                if (!P.both || p < q) {
+                    csum += t[i].z;
+                    ccnt += 1;
+                }
             }
         }
         ccnt = warp_sum(ccnt);
@@ -381,7 +457,8 @@ __device__ __forceinline__ bool crowded(const Params& P, long long live, long lo
 // every CTA samples its own worklist evenly, then every CTA ranks the same
 // samples (identical result everywhere).  INT_MAX: no useful split.  All
 // threads of all CTAs must call it (one grid barrier).
-__device__ __forceinline__ int split_threshold(const Params& P, const CompactSrc& S, long long live,
+template <class CSRC>
+__device__ __forceinline__ int split_threshold(const Params& P, const CSRC& S, long long live,
                                                long long winners, cg::grid_group& grid, int* s_w) {
     const int tid = threadIdx.x;
     const int ks = max(1, kSplitSamples / P.G);
@@ -389,7 +466,7 @@ __device__ __forceinline__ int split_threshold(const Params& P, const CompactSrc
     if ((int)blockIdx.x < ctas)
     for (int i = tid; i < ks; i += kBlock) {
         int w = INT_MAX;   // an empty arena votes "heavy"
-        if (S.cnt > 0) w = __ldcg(&S.base[(long long)(2 * i + 1) * S.cnt / (2 * ks)].z);
+        if (S.cnt > 0) w = tld_w<CSRC::SOA>(S.base, (long long)(2 * i + 1) * S.cnt / (2 * ks), P.wlcap);
         P.samp[blockIdx.x * ks + i] = w;
     }
     grid.sync();
@@ -516,7 +593,9 @@ __device__ __forceinline__ long long relabel(const Params& P, long long base, lo
     return tot;
 }
 
-template <int PH>
+// SOA: opts.tuple_layout 1; DRIVE: opts.drive (compile-time, so the default
+// instantiation carries none of the de-optimisations' code or registers)
+template <int PH, bool SOA = false, int DRIVE = 0>
 __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
     cg::grid_group grid = cg::this_grid();
     __shared__ int s_out, s_def;
@@ -538,9 +617,14 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
     }
     stamp(P, 4 + 2 * g);                      // populate done
     const int b = blockIdx.x;
-    int4* wl[2] = {P.wl0 + (long long)b * P.cap, P.wl1 + (long long)b * P.cap};
+    int4* wl[2] = {tadd<SOA>(P.wl0, (long long)b * P.cap), tadd<SOA>(P.wl1, (long long)b * P.cap)};
+    // opts.drive 1, "Topology-Driven": every pass A reads the phase's
+    // whole edge list again (the populate output, never overwritten: pass A
+    // always writes buffer 1) instead of the last round's survivors
+    constexpr bool topo = DRIVE == 1;
+    constexpr bool vc = DRIVE == 2;
     // the populate output of this CTA: regions w = b, b + G, ... (region mode)
-    const RegionSrc R = region_src(P, b, s_pre, s_rcnt, s_red, &st->live[g], PH == 1);
+    const RegionSrcT<SOA> R = region_src<SOA>(P, b, s_pre, s_rcnt, s_red, &st->live[g], PH == 1);
     if (b0 && tid == 0 && PH == 2) st->phase2_round = g;
     trace_cta(P, 4 + 2 * g);
     grid.sync();
@@ -550,7 +634,7 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
     int cur = 0;
     bool overflow = false;
     long long L = __ldcg(&st->live[g]);
-    CompactSrc C = compact_src(wl[0], 0);
+    CompactSrcT<SOA> C = compact_src<SOA>(wl[0], 0);
     // deferred tuples of a crowded-round split: at the back of this CTA's
     // arena in buffer hb (-1: none pending), hcnt of them (per CTA; hb is the
     // same in every CTA because every split decision is)
@@ -631,29 +715,41 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
         // the deferred set is then one run, drained together (any union of
         // deferred parts is heavier than the light part still running)
         int T = INT_MAX;
-        if constexpr (std::is_same<std::decay_t<decltype(S)>, CompactSrc>::value) {
+        if constexpr (is_compact_src<std::decay_t<decltype(S)>>::value) {
             if (!mapped && (hb < 0 || hb == (cur ^ 1)) && crowded(P, L, win, g)) {
                 T = split_threshold(P, S, L, win, grid, s_w);
                 if (tid == 0) s_def = hb < 0 ? 0 : hcnt;
                 __syncthreads();
             }
         }
-        if (T != INT_MAX) passA<true>(P, D, S, wl[cur ^ 1], &s_out, guard, T, wl[cur ^ 1] + P.cap, &s_def);
+        unsigned long long* const vcnt = &P.in->vc_cnt[g % 3];
+        if constexpr (vc) {
+            if (b0 && tid == 0) P.in->vc_cnt[(g + 1) % 3] = 0;   // next round's list counter (read 2 rounds ago)
+            passA_vc<PH, SOA>(P, D, vcnt, guard);
+        } else if constexpr (topo) {
+            passA(P, D, R, wl[1], &s_out, guard);
+        } else if (T != INT_MAX)
+            passA<true>(P, D, S, wl[cur ^ 1], &s_out, guard, T, tadd<SOA>(wl[cur ^ 1], P.cap), &s_def);
         else if (mapped) passA<false, true>(P, D, S, wl[cur ^ 1], &s_out, guard);
         else passA(P, D, S, wl[cur ^ 1], &s_out, guard);
-        cur ^= 1;
+        cur = topo ? 1 : cur ^ 1;
         __syncthreads();
-        C = compact_src(wl[cur], s_out);
+        C = compact_src<SOA>(wl[cur], s_out);
         if (T != INT_MAX) {
             hb = cur;
             hcnt = s_def;
             if (b0 && tid == 0) atomicAdd(&P.in->splits, 1);
         }
-        if (tid == 0 && C.cnt) atomicAdd(reinterpret_cast<unsigned long long*>(&st->live[g]), (unsigned long long)C.cnt);
+        if (!vc && tid == 0 && C.cnt) atomicAdd(reinterpret_cast<unsigned long long*>(&st->live[g]), (unsigned long long)C.cnt);
         trace_cta(P, 4 + 2 * g);
         grid.sync();
         stamp(P, 4 + 2 * g);
-        L = __ldcg(&st->live[g]);
+        if (vc) {
+            L = (long long)__ldcg(vcnt);
+            if (b0 && tid == 0) st->live[g] = L;
+        } else {
+            L = __ldcg(&st->live[g]);
+        }
         return true;
     };
     // the light part of a split is done: filter the deferred tuples (find,
@@ -664,7 +760,7 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
             overflow = true;
             return false;
         }
-        const CompactSrc H = compact_src(wl[hb] + P.cap - hcnt, hcnt);
+        const CompactSrcT<SOA> H = compact_src<SOA>(tadd<SOA>(wl[hb], P.cap - hcnt), hcnt);
         const int ob = hb ^ 1;
         hb = -1;
         hcnt = 0;
@@ -674,7 +770,7 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
         passA(P, D, H, wl[ob], &s_out, true);
         cur = ob;
         __syncthreads();
-        C = compact_src(wl[cur], s_out);
+        C = compact_src<SOA>(wl[cur], s_out);
         if (tid == 0 && C.cnt) atomicAdd(reinterpret_cast<unsigned long long*>(&st->live[g]), (unsigned long long)C.cnt);
         trace_cta(P, 4 + 2 * g);
         grid.sync();
@@ -685,7 +781,11 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
     if (L > 0 && round(R)) {
         for (;;) {
             if (L > 0) {
-                if (!round(C)) break;
+                if constexpr (vc) {
+                    if (!round(global_src<SOA>(P.wl1, L))) break;
+                } else {
+                    if (!round(C)) break;
+                }
             } else if (hb >= 0) {
                 if (!drain()) break;
             } else {

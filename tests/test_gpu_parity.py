@@ -115,6 +115,12 @@ def test_config_small(eclmst, name):
     dict(relabel=1), dict(relabel=0), dict(relabel=1, refilter=1), dict(relabel=1, giant_bitmap=1),
     dict(relabel=1, max_ctas=3), dict(relabel=1, path_halving=0), dict(relabel=1, filter=0),
     dict(relabel=1, refilter=1, filter=1, filter_c=1, giant_bitmap=1), dict(relabel=1, atomic_guards=1),
+    # the Table-5 de-optimisations, one at a time and all together
+    dict(populate_mode=1), dict(both_directions=1), dict(tuple_layout=1), dict(drive=1), dict(drive=2),
+    dict(populate_mode=1, both_directions=1, tuple_layout=1, drive=2, atomic_guards=0, filter=0, path_halving=0,
+         flatten=0),
+    dict(tuple_layout=1, refilter=1, relabel=1, giant_bitmap=1), dict(both_directions=1, refilter=1, relabel=1),
+    dict(drive=1, tuple_layout=1, both_directions=1), dict(populate_mode=1, relabel=1, max_ctas=3),
 ])
 @pytest.mark.parametrize("name", ["rmat", "uniform", "road"])
 def test_knobs_give_identical_msf(eclmst, name, opts):
@@ -298,6 +304,25 @@ def oracle_canonical(g):
     idx = g.nindex.numpy()
     rows = np.repeat(np.arange(g.n), np.diff(idx))
     return rows < g.nlist.numpy()
+
+
+DEOPTS = [dict(populate_mode=1), dict(both_directions=1), dict(tuple_layout=1), dict(drive=1), dict(drive=2),
+          dict(populate_mode=1, both_directions=1, tuple_layout=1, drive=2)]
+
+
+@pytest.mark.parametrize("opts", DEOPTS)
+@pytest.mark.parametrize("seed", range(6))
+def test_deopts_adversarial(eclmst, opts, seed):
+    """Every de-optimisation of Table 5 (NEXT-2) on tie-heavy multigraphs with
+    loops, both filter settings, a star row and a monotone path."""
+    kinds = ["ties", "two", "equal", "full", "uniform", "ties"]
+    g = G.random_small(300 + 97 * seed, 4000 + 500 * seed, seed=5000 + seed, weights=kinds[seed], multi=True,
+                       self_loops=True)
+    for filt in (-1, 0, 1):
+        assert_parity(eclmst, g, filter=filt, **opts)
+    if seed == 0:
+        assert_parity(eclmst, G.star_graph(5000, seed=1), **opts)
+        assert_parity(eclmst, G.path_graph(3000), **opts)
 
 
 @pytest.mark.parametrize("seed", range(12))
