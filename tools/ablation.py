@@ -4,9 +4,11 @@
   python tools/ablation.py --seeds 99 --configs rmat rgg --out profiles/r01_seeds.json
 
 Ablation: every option knob of ecl_mst_options that the paper evaluates as an
-optimisation (Table 5 semantics): atomic guards, the
-filter, path halving / flatten, the populate chunk order, the
-crowded-round split and the threshold constant c.  Each variant's mask and
+optimisation (Table 5 semantics): atomic guards, thread-
+based populate, the filter, path halving / flatten,
+both edge directions, no tuples, topology-driven and
+vertex-centric -- alone and cumulatively -- plus this build's own
+knobs (populate chunk order, crowded-round split, c, contraction).  Each variant's mask and
 total must equal the default run's bit for bit (the default is itself checked
 against the oracle by tests/ and bench.py); the JSON keeps the median time of
 `--runs` timed runs (CUDA events, L2 flushed before each).
@@ -44,6 +46,28 @@ VARIANTS = [
     ("filter c=3", {"filter_c": 3}),
     ("paper: 20 samples", {"threshold_samples": 20}),
     ("paper-like: 20 samples, no split", {"threshold_samples": 20, "refilter": 0}),
+    ("exact-quantile threshold", {"threshold_mode": 2}),
+    ("no contraction (relabel off)", {"relabel": 0}),
+    # Table 5: each de-optimisation alone ...
+    ("thread-based populate (P:372)", {"populate_mode": 1}),
+    ("both edge directions (P:375)", {"both_directions": 1}),
+    ("no tuples / SoA (P:376)", {"tuple_layout": 1}),
+    ("topology-driven (P:377)", {"drive": 1}),
+    ("vertex-centric (P:378)", {"drive": 2}),
+    # ... and cumulatively, in the paper's order.  Step (4), "no
+    # implicit path compression", has no knob of its own: pass B's hook needs
+    # the round's representatives in the tuples; the topology-
+    # driven step finds from the original endpoints in every round instead.
+    ("cum: no guards", {"atomic_guards": 0}),
+    ("cum: + thread-based", {"atomic_guards": 0, "populate_mode": 1}),
+    ("cum: + no filter", {"atomic_guards": 0, "populate_mode": 1, "filter": 0}),
+    ("cum: + both directions", {"atomic_guards": 0, "populate_mode": 1, "filter": 0, "both_directions": 1}),
+    ("cum: + no tuples", {"atomic_guards": 0, "populate_mode": 1, "filter": 0, "both_directions": 1,
+                          "tuple_layout": 1}),
+    ("cum: + topology-driven", {"atomic_guards": 0, "populate_mode": 1, "filter": 0, "both_directions": 1,
+                                "tuple_layout": 1, "drive": 1}),
+    ("cum: + vertex-centric", {"atomic_guards": 0, "populate_mode": 1, "filter": 0, "both_directions": 1,
+                               "tuple_layout": 1, "drive": 2}),
 ]
 
 
@@ -71,7 +95,8 @@ def ablation(cfgs, runs):
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
     for c in cfgs:
         g = synth.make_config(c, "full", device=dev)
-        ws = torch.empty(eclmst.ecl_mst_workspace_bytes(g.n, g.M), dtype=torch.uint8, device=dev)
+        ws = torch.empty(eclmst.ecl_mst_workspace_bytes(g.n, g.M, eclmst.default_options(both_directions=1)),
+                         dtype=torch.uint8, device=dev)
         rows = []
         ref_mask = ref_total = None
         for name, kw in VARIANTS:
