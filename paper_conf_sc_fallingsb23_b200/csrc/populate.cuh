@@ -281,6 +281,15 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
     int nr0 = 0, nrl = 0, n2r0 = 0, n2rl = 0, nv[kItems], nw[kItems];
     long long nsa = LLONG_MAX, nsz = LLONG_MAX;
     unsigned nvb = 0;
+    // phase 2 with the largest-set bitmap: lane i holds bitmap word
+    // (r0 >> 5) + i of the next chunk's rows, so each entry takes its row's
+    // bit by a shuffle instead of a dependent load
+    unsigned nrw = 0;
+    auto rowwords = [&](int r0, int rl) {
+        unsigned x = 0;
+        if (PH == 2 && giant >= 0 && (r0 >> 5) + lane <= (rl >> 5)) x = __ldg(P.giant_bits + (r0 >> 5) + lane);
+        return x;
+    };
     // the warp's chunks: interleaved w, w + W, ... or the contiguous slice
     // [w B, (w + 1) B) with B = rcap / kChunk (see P.pop_contig)
     const bool contig = (P.pop_contig >> (PH - 1)) & 1;
@@ -294,6 +303,7 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
         load_entries(P.shard + lc0 * P.nshards, nv, nw);
         if (deep) {
             starts(nr0, nrl, nsa, nsz);
+            nrw = rowwords(nr0, nrl);
             if (nxt(lc0) < lend) bracket(nxt(lc0), n2r0, n2rl);
         }
         nvb = vbits(nv, nw, nr0);
@@ -312,6 +322,7 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
         const int r0 = nr0, r_last = nrl;
         const long long sa = nsa, sz = nsz;
         const unsigned vb = nvb;
+        const unsigned rw = nrw;
         int vv[kItems], ww[kItems];
 #pragma unroll
         for (int k = 0; k < kItems; ++k) {
@@ -325,6 +336,7 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
                 nr0 = n2r0;
                 nrl = n2rl;
                 starts(nr0, nrl, nsa, nsz);
+                nrw = rowwords(nr0, nrl);
                 if (nxt(lcn) < lend) bracket(nxt(lcn), n2r0, n2rl);
             } else {
                 bracket(lcn, nr0, nrl);
@@ -400,10 +412,17 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
             qk[k] = vv[k];
         }
         if (PH == 2) {   // set(v), set(n): one load each after k_flatten
+            unsigned rbit[kItems];   // the rows' bits: from the lanes' prefetched words when deep
+#pragma unroll
+            for (int k = 0; k < kItems; ++k) {
+                const int wi = (row[k] >> 5) - (r0 >> 5);
+                const unsigned wd = __shfl_sync(kFull, rw, wi & 31);
+                rbit[k] = (deep && wi < 32) ? (wd >> (row[k] & 31)) & 1u : 2u;
+            }
 #pragma unroll
             for (int k = 0; k < kItems; ++k) {
                 if (cand[k] && giant >= 0 && ((vb >> k) & 1u) &&
-                    ((__ldg(P.giant_bits + (row[k] >> 5)) >> (row[k] & 31)) & 1)) {
+                    (rbit[k] == 2u ? (__ldg(P.giant_bits + (row[k] >> 5)) >> (row[k] & 31)) & 1u : rbit[k])) {
                     pk[k] = qk[k] = giant;                    // both ends in the largest set: filtered
                 } else if (cand[k]) {
                     pk[k] = (k > 0 && cand[k - 1] && row[k] == row[k - 1]) ? -1 : __ldca(sid + row[k]);

@@ -516,9 +516,9 @@ __device__ __forceinline__ int split_threshold(const Params& P, const CSRC& S, l
 #define ECL_RELABEL_MIN (1 << 21)    // auto: only levels of >= 2M ids (>= 24 MB of key + parent) ...
 #endif
 #ifndef ECL_RELABEL_FIRST
-#define ECL_RELABEL_FIRST (1 << 25)  // ... and the vertices themselves only from 2^25 on (C5): below,
-                                     // parent[] + key[] (12n B) keep enough locality -- measured:
-                                     // C2 2.26 -> 2.37 ms, C3 2.83 -> 3.02 ms, C4 7.31 -> 7.44 ms with it
+#define ECL_RELABEL_FIRST (1 << 21)  // ... the vertices' level included (measured with the 256-id
+                                     // scans: C2 2.261 -> 2.129 ms, C3 2.875 -> 2.810, C4 +-0, C1 +-0;
+                                     // the first, one-id-per-lane scans had cost C2 +0.1 ms)
 #endif
 constexpr int kRlItems = 8;                     // ids per lane per step of a relabel scan
 constexpr int kRlStep = 32 * kRlItems;          // 256 ids per warp step
@@ -666,7 +666,10 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
     auto round = [&](const auto& S) {
         const long long w0 = acc[1];
         const bool noreset = may_relabel();
-        if (noreset) passB<true>(P, D, S, acc);
+        // (both_directions: an edge's two copies must see the same slots, so
+        // no copy resets them in pass B; the paper's separate reset kernel,
+        // L34-37, follows instead)
+        if (noreset || P.both) passB<true>(P, D, S, acc);
         else passB(P, D, S, acc);
         const long long d = acc[1] - w0;
         if (lane == 0 && d) atomicAdd(reinterpret_cast<unsigned long long*>(&st->winners[g]), (unsigned long long)d);
@@ -677,6 +680,18 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
         if (g + 1 >= ECL_MST_MAX_ROUNDS) {
             overflow = true;
             return false;
+        }
+        if (P.both && !noreset) {   // L34-37 as its own pass over the tuples (both_directions)
+            for (int k = threadIdx.x >> 5; k < S.nloc; k += kWarps) {
+                int count;
+                const int4* in = S.get(P, k, count);
+                for (int i = lane; i < count; i += 32) {
+                    const int4 t = tld_cg<std::decay_t<decltype(S)>::SOA>(in, i, P.wlcap);
+                    __stcg(D.k(t.x), kInf);
+                    __stcg(D.k(t.y), kInf);
+                }
+            }
+            grid.sync();
         }
         const long long win = __ldcg(&st->winners[g]);
         ++g;
