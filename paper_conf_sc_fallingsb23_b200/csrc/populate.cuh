@@ -293,7 +293,7 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
     // the warp's chunks: interleaved w, w + W, ... or the contiguous slice
     // [w B, (w + 1) B) with B = rcap / kChunk (see P.pop_contig)
     const bool contig = (P.pop_contig >> (PH - 1)) & 1;
-    const long long span = P.rcap / kChunk;
+    const long long span = P.rcap / kChunk / (BOTH ? 2 : 1);   // chunks per warp (regions hold 2 copies)
     const long long step = contig ? 1 : P.W;
     const long long lc0 = contig ? (long long)w * span : w;
     const long long lend = contig ? min(lc0 + span, P.nlocal) : P.nlocal;
