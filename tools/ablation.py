@@ -89,7 +89,7 @@ def timed(g, opts, runs, ws, flush):
     return statistics.median(ts), mask, int(total.item()), eclmst.ecl_mst_read_stats(ws)
 
 
-def ablation(cfgs, runs):
+def ablation(cfgs, runs, path=None):
     out = {}
     dev = torch.device("cuda:0")
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
@@ -100,7 +100,12 @@ def ablation(cfgs, runs):
         rows = []
         ref_mask = ref_total = None
         for name, kw in VARIANTS:
-            ms, mask, total, st = timed(g, eclmst.default_options(**kw), runs, ws, flush)
+            try:
+                ms, mask, total, st = timed(g, eclmst.default_options(**kw), runs, ws, flush)
+            except Exception as e:   # (recorded, not fatal: e.g. a de-optimisation too slow or too large)
+                rows.append({"variant": name, "options": kw, "error": str(e)[:200]})
+                print(f"{c:8s} {name:34s} ERROR {e}", flush=True)
+                continue
             if ref_mask is None:
                 ref_mask, ref_total = mask.clone(), total
                 same = True
@@ -111,6 +116,9 @@ def ablation(cfgs, runs):
                          "sum_live": int(sum(st["live"]))})
             print(f"{c:8s} {name:34s} {ms:9.3f} ms  same={same} rounds={st['rounds']}", flush=True)
         out[c] = {"graph": g.name, "n": g.n, "M": g.M, "rows": rows}
+        if path:
+            with open(path, "w") as f:
+                json.dump(out, f, indent=1)
         del ws, g
         torch.cuda.empty_cache()
     return out
@@ -171,7 +179,8 @@ def main():
     ap.add_argument("--seeds", type=int, default=0, help="run the seed study with this many seeds instead")
     ap.add_argument("--out", default=None)
     args = ap.parse_args()
-    res = seed_study(args.configs, args.seeds, max(1, args.runs)) if args.seeds else ablation(args.configs, args.runs)
+    res = (seed_study(args.configs, args.seeds, max(1, args.runs)) if args.seeds
+           else ablation(args.configs, args.runs, args.out))
     res["gpu"] = torch.cuda.get_device_name(0)
     if args.out:
         with open(args.out, "w") as f:
