@@ -115,6 +115,11 @@ typedef struct ecl_mst_options {
     int32_t drive;           /* 0 (default) data-driven worklist; 1 "Topology-Driven": every
                                 round processes all edges of the phase again; 2 "Vertex-Centric"
                                 (P:378): topology-driven with one thread per vertex and its row */
+    int32_t dist_loop;       /* sharded path only: 0 (default) host-driven rounds, NCCL allreduce(min)
+                                per round; 1 device-initiated: one persistent kernel per phase runs
+                                every round (exchange = a device-side min over the shards' key
+                                arrays, rep passes, compaction, pass A) with no host round-trip;
+                                local (virtual) shards only in this build (world 1) */
 } ecl_mst_options;
 
 /* per-run statistics written by the device into the workspace */

@@ -47,6 +47,7 @@ class EclMstOptions(ctypes.Structure):
         ("both_directions", ctypes.c_int32),
         ("tuple_layout", ctypes.c_int32),
         ("drive", ctypes.c_int32),
+        ("dist_loop", ctypes.c_int32),
     ]
 
 

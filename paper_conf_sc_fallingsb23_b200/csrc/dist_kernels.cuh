@@ -364,4 +364,188 @@ __global__ void __launch_bounds__(kBlock, 2) k_dist_drain(Params P, int g, int h
     }
 }
 
+// ===========================================================================
+// Device-initiated sharded round loop (opts.dist_loop 1; SURVEY §8(f)
+// NEXT-4).  One cooperative kernel runs every round of a phase -- the key
+// exchange, the rep passes, the root-list compaction and every shard's pass
+// A -- with grid barriers between the stages and no host involvement: the
+// termination test ("no set has a finite key") is a grid-wide count that
+// every CTA reads.  The exchange is a device-side reduction: each reduced
+// key is the min over the key arrays of all shards this GPU can address
+// (Params::keys_all; with virtual shards these are local arrays, with peer
+// ranks they would be their NVLink-mapped arrays).  Same data flow and same
+// decisions as the host loop of ecl_mst_dist_device, so the partition, the
+// round count and the MSF are identical.
+// ===========================================================================
+struct DistLoop {
+    const Params* sps;        // device copy of every local shard's Params
+    int S;                    // local shards
+    int g0;                   // first global round of this phase
+    const int* R0;            // first root list (nullptr: all n vertices)
+    long long nR0;
+    int* rl[2];               // root-list buffers
+    long long* buf;           // reduced keys of the current root list
+    unsigned char* keep;      // rep pass 2: the set stays in the next list
+    int* bcnt;                // per CTA: kept sets of its slice
+    unsigned long long* found;   // [2]: sets with a finite key, per round parity
+};
+
+// order-preserving compaction of R by keep over the cooperative grid (every
+// CTA a contiguous slice); returns the new size (same in every CTA)
+__device__ __forceinline__ long long dl_compact(const int* R, long long nR, const unsigned char* keep, int* bcnt,
+                                                int* out, cg::grid_group& grid, int* s_w) {
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const long long lo = nR * blockIdx.x / gridDim.x, hi = nR * (blockIdx.x + 1) / gridDim.x;
+    const long long per = (hi - lo + kWarps - 1) / kWarps;
+    const long long wlo = min(hi, lo + warp * per), whi = min(hi, wlo + per);
+    int c = 0;
+    for (long long i = wlo + lane; i < whi; i += 32) c += keep[i];
+    c = warp_sum(c);
+    if (lane == 0) s_w[warp] = c;
+    __syncthreads();
+    if (tid == 0) {
+        int t = 0;
+        for (int w = 0; w < kWarps; ++w) t += s_w[w];
+        bcnt[blockIdx.x] = t;
+    }
+    grid.sync();
+    long long base = 0, tot = 0;
+    for (unsigned k = 0; k < gridDim.x; ++k) {   // (every thread: gridDim.x <= a few hundred)
+        const long long v = __ldcg(bcnt + k);
+        tot += v;
+        if (k < blockIdx.x) base += v;
+    }
+    for (int w = 0; w < warp; ++w) base += s_w[w];
+    const unsigned lt = (1u << lane) - 1u;
+    for (long long i0 = wlo; i0 < whi; i0 += 32) {
+        const long long i = i0 + lane;
+        const bool k = i < whi && keep[i];
+        const unsigned m = __ballot_sync(kFull, k);
+        if (k) out[base + __popc(m & lt)] = (int)set_of(R, i);
+        base += __popc(m);
+    }
+    grid.sync();
+    return tot;
+}
+
+template <int PH>
+__global__ void __launch_bounds__(kBlock, 2) k_dist_loop(Params P0, DistLoop DL) {
+    cg::grid_group grid = cg::this_grid();
+    __shared__ int s_out, s_w[kWarps];
+    __shared__ long long s_red[3][kWarps];
+    __shared__ int s_pre[kMaxRegionsPerCta + 1];
+    __shared__ int s_rcnt[kMaxRegionsPerCta];
+    const int tid = threadIdx.x, lane = tid & 31;
+    const int b = blockIdx.x;
+    const bool b0 = b == 0;
+    const long long gstride = (long long)gridDim.x * kBlock;
+    const long long gtid = (long long)b * kBlock + tid;
+    ecl_mst_stats* st = P0.st;
+    if (!input_ok(P0) || (PH == 2 && !phase2_needed(P0))) return;
+    int g = DL.g0;
+    const int* R = DL.R0;
+    long long nR = DL.nR0;
+    int rb = 0;
+    int cur = 0;
+    bool first = true;
+    for (;;) {
+        // ---- exchange: reduced best-edge key of every set of R ----
+        for (long long i = gtid; i < nR; i += gstride) {
+            const long long x = set_of(R, i);
+            long long m = kInf;
+            for (int s2 = 0; s2 < P0.nkeys; ++s2) m = min(m, __ldcg(P0.keys_all[s2] + x));
+            DL.buf[i] = m;
+        }
+        grid.sync();
+        for (long long i = gtid; i < nR; i += gstride) P0.key[set_of(R, i)] = DL.buf[i];   // (shard 0: by set id)
+        grid.sync();
+        // ---- rep pass 1: the other end of every set's lightest edge, mutual? ----
+        const DS D = ds_of(P0);
+        for (long long i = gtid; i < nR; i += gstride) {
+            const long long kx = DL.buf[i];
+            if (kx == kInf) continue;
+            const long long x = set_of(R, i);
+            const unsigned j = (unsigned)(kx & 0xffffffffll);
+            const int u = row_of_entry(P0, (long long)j);
+            const int v = __ldg(P0.nlist + j);
+            const int pu = find_root(D, u, false), pv = find_root(D, v, false);
+            const int q = (pu == (int)x) ? pv : pu;
+            P0.tgt[i] = q | (__ldcg(P0.key + q) == kx ? (int)0x80000000 : 0);
+        }
+        grid.sync();
+        // ---- rep pass 2 (L30-31, L34-37): hook, mark, sum, reset ----
+        {
+            long long wsum = 0, wcnt = 0;
+            unsigned long long found = 0;
+            for (long long i = gtid; i < nR; i += gstride) {
+                const long long kx = DL.buf[i];
+                const long long x = set_of(R, i);
+                if (kx == kInf) {
+                    DL.keep[i] = 0;
+                    continue;
+                }
+                ++found;
+                const int t = P0.tgt[i];
+                const int q = t & 0x7fffffff;
+                const bool mutual = t < 0;
+                if (!mutual || (int)x > q) P0.parent[x] = q;
+                if (!mutual || (int)x < q) {
+                    P0.in_mst[(unsigned)(kx & 0xffffffffll)] = 1;
+                    wsum += (int)(kx >> 32);
+                    wcnt += 1;
+                }
+                DL.keep[i] = mutual && (int)x < q;
+                for (int s2 = 0; s2 < P0.nkeys; ++s2) P0.keys_all[s2][x] = kInf;
+            }
+            wsum = warp_sum(wsum);
+            wcnt = warp_sum(wcnt);
+            found = warp_sum(found);
+            if (lane == 0 && found) atomicAdd(&DL.found[g & 1], found);
+            if (lane == 0 && wcnt) {
+                atomicAdd(reinterpret_cast<unsigned long long*>(&st->total_weight), (unsigned long long)wsum);
+                atomicAdd(reinterpret_cast<unsigned long long*>(&st->msf_edges), (unsigned long long)wcnt);
+                atomicAdd(reinterpret_cast<unsigned long long*>(&st->winners[g]), (unsigned long long)wcnt);
+            }
+        }
+        grid.sync();
+        const unsigned long long nfound = __ldcg(&DL.found[g & 1]);
+        if (b0 && tid == 0) DL.found[(g + 1) & 1] = 0;   // next round's counter (its last reader was round g - 1)
+        if (nfound == 0) break;                          // no set has a live edge anywhere: the phase is done
+        if (g + 1 >= ECL_MST_MAX_ROUNDS) {
+            if (b0 && tid == 0) atomicExch(&st->status, ECL_MST_ERR_ROUNDS);
+            break;
+        }
+        // ---- the next root list: the roots that kept a live edge ----
+        int* const Rn = DL.rl[rb];
+        const long long nRn = dl_compact(R, nR, DL.keep, DL.bcnt, Rn, grid, s_w);
+        // ---- pass A of round g + 1 on every local shard ----
+        ++g;
+        for (int k = 0; k < DL.S; ++k) {
+            const Params& Pk = DL.sps[k];
+            if (b >= Pk.G) continue;
+            int4* wl[2] = {Pk.wl0 + (long long)b * Pk.cap, Pk.wl1 + (long long)b * Pk.cap};
+            if (tid == 0) s_out = 0;
+            __syncthreads();
+            if (first) {
+                const RegionSrc RS = region_src(Pk, b, s_pre, s_rcnt, s_red, &st->live[g - 1], g - 1 == 0);
+                passA(Pk, ds_of(Pk), RS, wl[cur ^ 1], &s_out, Pk.guards != 0);
+            } else {
+                passA(Pk, ds_of(Pk), compact_src(wl[cur], Pk.acnt[b]), wl[cur ^ 1], &s_out, Pk.guards != 0);
+            }
+            __syncthreads();
+            if (tid == 0) {
+                Pk.acnt[b] = s_out;
+                if (s_out) atomicAdd(reinterpret_cast<unsigned long long*>(&st->live[g]), (unsigned long long)s_out);
+            }
+        }
+        grid.sync();
+        cur ^= 1;
+        first = false;
+        R = Rn;
+        nR = nRn;
+        rb ^= 1;
+    }
+    if (b0 && tid == 0) P0.in->g_end = g;
+}
+
 }  // namespace eclmst

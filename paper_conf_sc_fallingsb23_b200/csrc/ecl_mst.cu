@@ -139,6 +139,7 @@ void ecl_mst_default_options(ecl_mst_options* o) {
     o->both_directions = 0;
     o->tuple_layout = 0;
     o->drive = 0;
+    o->dist_loop = 0;
 }
 
 size_t ecl_mst_workspace_bytes(int64_t n, int64_t M) {
@@ -740,7 +741,7 @@ static void release(DistHandle* h) {
 
 struct DistLayout {
     size_t stats, internal, rowstart, parent, tgt, keyptrs, rl0, rl1, rbuf, keep, bcnt, dsplit, giant, qhist, setid,
-        shard0, shard_bytes, total;
+        sps, found, shard0, shard_bytes, total;
     size_t region, acnt, hcnt, key, wl0, wl1;   // offsets inside one shard block
     long long wl_cap, nlocal_max;
 };
@@ -768,6 +769,8 @@ static inline DistLayout dist_layout(int64_t n, int64_t M, int S, int world) {
     L.giant = off;    off = align_up(off + sizeof(unsigned) * (size_t)((n + 31) / 32 + 1), 256);   // largest-set bitmap
     L.qhist = off;    off = align_up(off + sizeof(unsigned long long) * (size_t)kQBins, 256);
     L.setid = off;    off = align_up(off + sizeof(int) * (size_t)n, 256);
+    L.sps = off;      off = align_up(off + sizeof(Params) * (size_t)S, 256);   // dist_loop: the shards' Params
+    L.found = off;    off = align_up(off + 2 * sizeof(unsigned long long), 256);
     size_t so = 0;
     L.region = so; so = align_up(so + sizeof(int4) * (size_t)kMaxPopWarps, 256);
     L.acnt = so;   so = align_up(so + sizeof(int) * (size_t)kMaxGrid, 256);
@@ -898,7 +901,17 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
     // device from allreduced values, the same on every rank
     // (auto: only where the two-phase filter is on too, M >= 4n -- the dense
     // graphs whose giant set crowds the rounds; C2 x1 4.33 vs 3.80 ms with them)
-    const bool split_on = o.refilter > 0 || (o.refilter < 0 && (o.filter > 0 || (o.filter < 0 && M >= 4LL * n)));
+    const bool dloop = o.dist_loop != 0;
+    if (dloop && (world > 1 || h->comm))
+        return fail(ECL_MST_ERR_INVALID, "dist_loop 1 (device-initiated rounds) runs local shards only (world 1, no NCCL)");
+    // (the device loop has no crowded-round split: every split decision of
+    // the host loop rides on its allreduce)
+    const bool split_on = !dloop && (o.refilter > 0 || (o.refilter < 0 && (o.filter > 0 || (o.filter < 0 && M >= 4LL * n))));
+    int loop_occ = 0;
+    if (dloop) {
+        cudaError_t e0 = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&loop_occ, k_dist_loop<1>, kBlock, 0);
+        if (e0 != cudaSuccess || loop_occ < 1) return fail(ECL_MST_ERR_CUDA, "dist_loop occupancy");
+    }
     DistSplit* dsp = reinterpret_cast<DistSplit*>(ws + L.dsplit);
     // per-shard launch geometry and parameters
     std::vector<Params> sp(S);
@@ -911,7 +924,7 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
         std::memset(&P, 0, sizeof P);
         const int shard = rank * S + k;
         const long long nlocal = shard < nchunks ? (nchunks - shard + Pt - 1) / Pt : 0;
-        long long G = (long long)di.sms * di.occ;
+        long long G = (long long)di.sms * (dloop ? std::min(loop_occ, di.occ) : di.occ);   // (co-resident in the loop)
         if (G > std::max<long long>(nlocal, 1)) G = std::max<long long>(nlocal, 1);
         if (G > kMaxGrid) G = kMaxGrid;
         long long W = (long long)di.sms * di.pop_occ * kPopWarps;
@@ -954,7 +967,7 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
         P.halving = o.path_halving ? 1 : 0;
         P.guards = o.atomic_guards == 0 ? 0 : 1;
         P.flatten = o.flatten ? 1 : 0;
-        P.refilter = o.refilter < 0 ? -1 : (o.refilter ? 1 : 0);   // crowded-round split (Q17)
+        P.refilter = dloop ? 0 : (o.refilter < 0 ? -1 : (o.refilter ? 1 : 0));   // crowded-round split (Q17)
         P.round_bound = round_bound_for(n);
         P.samp = nullptr;
         P.qhist = reinterpret_cast<unsigned long long*>(ws + L.qhist);
@@ -1020,7 +1033,62 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
         k_dist_compact<<<cb, kCompactBlock, 0, s>>>(nullptr, n, rkeep, rcnt, out, &in->nroots, &in->reps, h->d_map,
                                                     nullptr);
     };
-    for (int ph = 1; ph <= 2; ++ph) {
+    if (dloop) {   // ---- device-initiated rounds: one persistent kernel per phase ----
+        Params* d_sps = reinterpret_cast<Params*>(ws + L.sps);
+        unsigned long long* d_found = reinterpret_cast<unsigned long long*>(ws + L.found);
+        e = cudaMemcpyAsync(d_sps, sp.data(), sizeof(Params) * S, cudaMemcpyHostToDevice, s);
+        if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "dist_loop params: %s", cudaGetErrorString(e));
+        long long Gl = 1;
+        for (int k = 0; k < S; ++k) Gl = std::max<long long>(Gl, sp[k].G);
+        auto run_loop = [&](int ph, int g0, const int* R0, long long nR0, int* r_a, int* r_b) -> int {
+            DistLoop DL;
+            DL.sps = d_sps;
+            DL.S = S;
+            DL.g0 = g0;
+            DL.R0 = R0;
+            DL.nR0 = nR0;
+            DL.rl[0] = r_a;
+            DL.rl[1] = r_b;
+            DL.buf = reinterpret_cast<long long*>(ws + L.rbuf);
+            DL.keep = rkeep;
+            DL.bcnt = rcnt;
+            DL.found = d_found;
+            cudaError_t e2 = cudaMemsetAsync(d_found, 0, 2 * sizeof(unsigned long long), s);
+            void* largs[] = {&P0, &DL};
+            if (e2 == cudaSuccess)
+                e2 = cudaLaunchCooperativeKernel(ph == 1 ? reinterpret_cast<const void*>(k_dist_loop<1>)
+                                                         : reinterpret_cast<const void*>(k_dist_loop<2>),
+                                                 dim3((unsigned)Gl), dim3(kBlock), largs, 0, s);
+            long long gend = 0;
+            if (e2 == cudaSuccess) e2 = cudaMemcpyAsync(h->h_pin, &in->g_end, sizeof(int), cudaMemcpyDeviceToHost, s);
+            if (e2 == cudaSuccess) e2 = cudaStreamSynchronize(s);   // (once per phase)
+            if (e2 != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "dist_loop: %s", cudaGetErrorString(e2));
+            std::memcpy(&gend, h->h_pin, sizeof(int));
+            g = (int)gend;
+            return ECL_MST_OK;
+        };
+        for (int k = 0; k < S; ++k) k_populate<1><<<(unsigned)ceil_div(sp[k].W, kPopWarps), kPopBlock, 0, s>>>(sp[k]);
+        if ((rc = check("populate"))) return rc;
+        if ((rc = run_loop(1, 0, nullptr, n, rlist[0], rlist[1]))) return rc;
+        long long filtered = 0, heavy = 0;
+        if ((rc = read_word(&st->heavy_edges, &heavy))) return rc;
+        if ((rc = read_word(&st->filtered, &filtered))) return rc;
+        if ((filtered & 0xffffffffll) && heavy != 0 && g + 1 < ECL_MST_MAX_ROUNDS) {
+            k_flatten<1><<<vblocks, 256, 0, s>>>(P0);
+            k_giant<<<1, 256, 0, s>>>(P0);
+            k_flatten<2><<<vblocks, 256, 0, s>>>(P0);
+            launch_roots(rlist[0]);
+            ++g;
+            e = cudaMemcpyAsync(&st->phase2_round, &g, sizeof(int), cudaMemcpyHostToDevice, s);
+            if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+            if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "phase2: %s", cudaGetErrorString(e));
+            const long long nroots = reinterpret_cast<volatile long long*>(h->h_map)[1];
+            for (int k = 0; k < S; ++k) k_populate<2><<<(unsigned)ceil_div(sp[k].W, kPopWarps), kPopBlock, 0, s>>>(sp[k]);
+            if ((rc = check("populate2"))) return rc;
+            if ((rc = run_loop(2, g, rlist[0], nroots, rlist[1], rlist[0]))) return rc;
+        }
+    }
+    for (int ph = 1; ph <= 2 && !dloop; ++ph) {
         if (ph == 2) {
             // the phase-2 decision needs the global deferred count
             if ((rc = allreduce(&st->canonical_edges, 2, kNcclSum))) return rc;

@@ -211,3 +211,65 @@ def test_virtual_shards_fuzz(ecl, seed):
             assert st["msf_edges"] == ocount, opts
     finally:
         ecl.ecl_mst_dist_finalize(h)
+
+
+# ---------------------------------------------- device-initiated round loop ---
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("shards", [1, 2, 3, 5])
+@pytest.mark.parametrize("name", list(synth.CONFIGS))
+def test_device_loop_parity(ecl, name, shards):
+    """opts.dist_loop 1 (NEXT-4): every round of a phase inside one persistent
+    kernel -- exchange (device-side min over the shards' key arrays), rep
+    passes, compaction, pass A -- bit-exact against the oracle."""
+    g = synth.make_config(name, "small")
+    h = ecl.ecl_mst_dist_init(None, 0, 1)
+    try:
+        mask, total, st = dist_run(ecl, g, h, shards, dist_loop=1)
+    finally:
+        ecl.ecl_mst_dist_finalize(h)
+    omask, ototal, ocount = oracle.kruskal_graph(g)
+    assert st["status"] == 0
+    assert total == ototal and np.array_equal(mask, omask)
+    assert st["msf_edges"] == ocount
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("seed", range(10))
+def test_device_loop_fuzz(ecl, seed):
+    kinds = ["ties", "two", "equal", "full", "uniform"]
+    n = 40 + 131 * seed
+    g = G.random_small(n, 7 * n + 13 * seed, seed=1900 + seed, weights=kinds[seed % 5], multi=True,
+                       self_loops=seed % 2 == 1)
+    omask, ototal, ocount = oracle.kruskal_graph(g)
+    h = ecl.ecl_mst_dist_init(None, 0, 1)
+    try:
+        for opts in (dict(), dict(filter=1, threshold_mode=1, threshold=0), dict(filter=0), dict(giant_bitmap=1),
+                     dict(filter=1, filter_c=1, max_ctas=3)):
+            mask, total, st = dist_run(ecl, g, h, 1 + seed % 4, dist_loop=1, **opts)
+            assert st["status"] == 0, opts
+            assert total == ototal and np.array_equal(mask, omask), opts
+            assert st["msf_edges"] == ocount, opts
+    finally:
+        ecl.ecl_mst_dist_finalize(h)
+
+
+@pytest.mark.gpu
+def test_device_loop_matches_host_loop_rounds(ecl):
+    """Same hook rule and data flow: the device loop's per-round winners, live
+    counts and round count equal the host-driven loop's and the single-GPU
+    kernel's (no crowded-round splits in either)."""
+    g = synth.make_config("rmat", "small")
+    gd = g.to("cuda:0")
+    _, _, ws = ecl.ecl_mst_device(gd.n, gd.nindex, gd.nlist, gd.eweight, options=ecl.default_options(refilter=0))
+    single = ecl.ecl_mst_read_stats(ws)
+    h = ecl.ecl_mst_dist_init(None, 0, 1)
+    try:
+        _, _, host = dist_run(ecl, g, h, 3, refilter=0)
+        _, _, dev = dist_run(ecl, g, h, 3, dist_loop=1)
+    finally:
+        ecl.ecl_mst_dist_finalize(h)
+    for st in (host, dev):
+        assert st["rounds"] == single["rounds"]
+        assert st["winners"] == single["winners"]
+        assert st["live"] == single["live"]
