@@ -359,8 +359,11 @@ def main():
         raise RuntimeError(f"generator drift: {(g.name, n, M)} != FULL_SIZES {fs[:3]}")
 
     handle = None
+    opt_kw0 = {k: int(v) for k, v in (o.split("=", 1) for o in args.opt)}
     if use_dist:   # edge-sharded path: NCCL allreduce(min) per round inside the library
-        handle = eclmst.dist.init_from_group()
+        # (the device-initiated round loop, dist_loop=1, runs without NCCL at world 1)
+        handle = (eclmst.ecl_mst_dist_init(None, 0, 1) if world == 1 and opt_kw0.get("dist_loop")
+                  else eclmst.dist.init_from_group())
         ws_bytes = eclmst.ecl_mst_dist_workspace_bytes(n, M, 1, world)
     else:
         ws_bytes = eclmst.ecl_mst_workspace_bytes(n, M)

@@ -448,6 +448,10 @@ __global__ void __launch_bounds__(kBlock, 2) k_dist_loop(Params P0, DistLoop DL)
     int rb = 0;
     int cur = 0;
     bool first = true;
+    // the populate output of every shard: its size (live[g0]) and, in phase
+    // 1, the canonical / deferred counts -- even if no round follows
+    for (int k = 0; k < DL.S; ++k)
+        if (b < DL.sps[k].G) region_src(DL.sps[k], b, s_pre, s_rcnt, s_red, &st->live[g], PH == 1);
     for (;;) {
         // ---- exchange: reduced best-edge key of every set of R ----
         for (long long i = gtid; i < nR; i += gstride) {
@@ -527,7 +531,7 @@ __global__ void __launch_bounds__(kBlock, 2) k_dist_loop(Params P0, DistLoop DL)
             if (tid == 0) s_out = 0;
             __syncthreads();
             if (first) {
-                const RegionSrc RS = region_src(Pk, b, s_pre, s_rcnt, s_red, &st->live[g - 1], g - 1 == 0);
+                const RegionSrc RS = region_src(Pk, b, s_pre, s_rcnt, s_red, nullptr, false);   // (counted above)
                 passA(Pk, ds_of(Pk), RS, wl[cur ^ 1], &s_out, Pk.guards != 0);
             } else {
                 passA(Pk, ds_of(Pk), compact_src(wl[cur], Pk.acnt[b]), wl[cur ^ 1], &s_out, Pk.guards != 0);

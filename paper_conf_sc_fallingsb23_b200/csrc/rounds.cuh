@@ -225,7 +225,7 @@ __device__ __forceinline__ RegionSrcT<SOA> region_src(const Params& P, int b, in
             canon += s_red[1][w2];
             heavy += s_red[2][w2];
         }
-        if (kept) atomicAdd(reinterpret_cast<unsigned long long*>(live_slot), (unsigned long long)kept);
+        if (kept && live_slot) atomicAdd(reinterpret_cast<unsigned long long*>(live_slot), (unsigned long long)kept);
         if (count_phase1) {
             if (canon) atomicAdd(reinterpret_cast<unsigned long long*>(&P.st->canonical_edges), (unsigned long long)canon);
             if (heavy) atomicAdd(reinterpret_cast<unsigned long long*>(&P.st->heavy_edges), (unsigned long long)heavy);
