@@ -456,25 +456,42 @@ __global__ void __launch_bounds__(kBlock, 2) k_dist_loop(Params P0, DistLoop DL)
         // ---- exchange: reduced best-edge key of every set of R ----
         for (long long i = gtid; i < nR; i += gstride) {
             const long long x = set_of(R, i);
-            long long m = kInf;
-            for (int s2 = 0; s2 < P0.nkeys; ++s2) m = min(m, __ldcg(P0.keys_all[s2] + x));
+            long long m = __ldcg(P0.keys_all[0] + x);
+            for (int s2 = 1; s2 < P0.nkeys; ++s2) m = min(m, __ldcg(P0.keys_all[s2] + x));
             DL.buf[i] = m;
         }
         grid.sync();
-        for (long long i = gtid; i < nR; i += gstride) P0.key[set_of(R, i)] = DL.buf[i];   // (shard 0: by set id)
-        grid.sync();
+        if (P0.nkeys > 1) {   // the reduced keys by set id, in shard 0's array (one shard: already there)
+            for (long long i = gtid; i < nR; i += gstride) P0.key[set_of(R, i)] = DL.buf[i];
+            grid.sync();
+        }
         // ---- rep pass 1: the other end of every set's lightest edge, mutual? ----
+        // (four sets per thread in flight: each is a chain of dependent loads)
         const DS D = ds_of(P0);
-        for (long long i = gtid; i < nR; i += gstride) {
-            const long long kx = DL.buf[i];
-            if (kx == kInf) continue;
-            const long long x = set_of(R, i);
-            const unsigned j = (unsigned)(kx & 0xffffffffll);
-            const int u = row_of_entry(P0, (long long)j);
-            const int v = __ldg(P0.nlist + j);
-            const int pu = find_root(D, u, false), pv = find_root(D, v, false);
-            const int q = (pu == (int)x) ? pv : pu;
-            P0.tgt[i] = q | (__ldcg(P0.key + q) == kx ? (int)0x80000000 : 0);
+        for (long long i0 = gtid; i0 < nR; i0 += 4 * gstride) {
+            long long kx[4];
+            unsigned j[4];
+            int u[4], v[4];
+#pragma unroll
+            for (int a = 0; a < 4; ++a) {
+                const long long i = i0 + a * gstride;
+                kx[a] = i < nR ? DL.buf[i] : kInf;
+                j[a] = (unsigned)(kx[a] & 0xffffffffll);
+            }
+#pragma unroll
+            for (int a = 0; a < 4; ++a) {
+                u[a] = kx[a] != kInf ? row_of_entry(P0, (long long)j[a]) : 0;
+                v[a] = kx[a] != kInf ? __ldg(P0.nlist + j[a]) : 0;
+            }
+#pragma unroll
+            for (int a = 0; a < 4; ++a) {
+                if (kx[a] == kInf) continue;
+                const long long i = i0 + a * gstride;
+                const long long x = set_of(R, i);
+                const int pu = find_root(D, u[a], false), pv = find_root(D, v[a], false);
+                const int q = (pu == (int)x) ? pv : pu;
+                P0.tgt[i] = q | (__ldcg(P0.key + q) == kx[a] ? (int)0x80000000 : 0);
+            }
         }
         grid.sync();
         // ---- rep pass 2 (L30-31, L34-37): hook, mark, sum, reset ----
