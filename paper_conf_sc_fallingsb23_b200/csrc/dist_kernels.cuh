@@ -393,7 +393,7 @@ struct DistLoop {
 // order-preserving compaction of R by keep over the cooperative grid (every
 // CTA a contiguous slice); returns the new size (same in every CTA)
 __device__ __forceinline__ long long dl_compact(const int* R, long long nR, const unsigned char* keep, int* bcnt,
-                                                int* out, cg::grid_group& grid, int* s_w) {
+                                                int* out, cg::grid_group& grid, int* s_w, long long (*s_red)[kWarps]) {
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const long long lo = nR * blockIdx.x / gridDim.x, hi = nR * (blockIdx.x + 1) / gridDim.x;
     const long long per = (hi - lo + kWarps - 1) / kWarps;
@@ -409,11 +409,23 @@ __device__ __forceinline__ long long dl_compact(const int* R, long long nR, cons
         bcnt[blockIdx.x] = t;
     }
     grid.sync();
-    long long base = 0, tot = 0;
-    for (unsigned k = 0; k < gridDim.x; ++k) {   // (every thread: gridDim.x <= a few hundred)
+    long long before = 0, total = 0;   // (the CTA counts: strided over the threads, then a block sum)
+    for (unsigned k = tid; k < gridDim.x; k += kBlock) {
         const long long v = __ldcg(bcnt + k);
-        tot += v;
-        if (k < blockIdx.x) base += v;
+        total += v;
+        if (k < blockIdx.x) before += v;
+    }
+    before = warp_sum(before);
+    total = warp_sum(total);
+    if (lane == 0) {
+        s_red[0][warp] = before;
+        s_red[1][warp] = total;
+    }
+    __syncthreads();
+    long long base = 0, tot = 0;
+    for (int w = 0; w < kWarps; ++w) {
+        base += s_red[0][w];
+        tot += s_red[1][w];
     }
     for (int w = 0; w < warp; ++w) base += s_w[w];
     const unsigned lt = (1u << lane) - 1u;
@@ -538,7 +550,7 @@ __global__ void __launch_bounds__(kBlock, 2) k_dist_loop(Params P0, DistLoop DL)
         }
         // ---- the next root list: the roots that kept a live edge ----
         int* const Rn = DL.rl[rb];
-        const long long nRn = dl_compact(R, nR, DL.keep, DL.bcnt, Rn, grid, s_w);
+        const long long nRn = dl_compact(R, nR, DL.keep, DL.bcnt, Rn, grid, s_w, s_red);
         // ---- pass A of round g + 1 on every local shard ----
         ++g;
         for (int k = 0; k < DL.S; ++k) {
