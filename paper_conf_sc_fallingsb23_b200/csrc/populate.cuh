@@ -194,10 +194,6 @@ template <int PH, bool SOA = false, bool BOTH = false>
 #endif
 __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) {
     __shared__ int s_mark[kPopWarps][kChunk];
-    // phase 2 with the largest-set bitmap: the chunk's surviving candidates
-    // (not filtered by the bitmap), packed so each is handled by one lane
-    __shared__ int4 s_sv[PH == 2 ? kPopWarps : 1][kChunk];
-    __shared__ unsigned char s_fl[PH == 2 ? kPopWarps : 1][kChunk];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     if (!input_ok(P)) return;   // k_init rejected nindex: rowstart[] is not valid
     if (PH == 2 && !phase2_needed(P)) return;
@@ -422,62 +418,6 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
                 const int wi = (row[k] >> 5) - (r0 >> 5);
                 const unsigned wd = __shfl_sync(kFull, rw, wi & 31);
                 rbit[k] = (deep && wi < 32) ? (wd >> (row[k] & 31)) & 1u : 2u;
-            }
-            if (!BOTH && giant >= 0) {
-                // Survivors: candidates with an end outside the largest set
-                // (about 5% of the heavy edges on C5).  Pack them into the
-                // warp's shared buffer and give each its own lane, so the
-                // set lookups, key records and the append run once per
-                // survivor instead of once per item slot of every lane.
-                unsigned fl[kItems];
-                bool sv[kItems];
-#pragma unroll
-                for (int k = 0; k < kItems; ++k) {
-                    const unsigned ub = cand[k] ? (rbit[k] == 2u ? (__ldg(P.giant_bits + (row[k] >> 5)) >> (row[k] & 31)) & 1u
-                                                                 : rbit[k]) : 0u;
-                    const unsigned vbk = (vb >> k) & 1u;
-                    fl[k] = ub | (vbk << 1);
-                    sv[k] = cand[k] && !(ub && vbk);
-                }
-                int4* const buf = s_sv[warp];
-                unsigned char* const fbuf = s_fl[warp];
-                const unsigned lt = (1u << lane) - 1u;
-                int nsv = 0;
-#pragma unroll
-                for (int k = 0; k < kItems; ++k) {
-                    const unsigned mk = __ballot_sync(kFull, sv[k]);
-                    if (sv[k]) {
-                        const int at = nsv + __popc(mk & lt);
-                        buf[at] = make_int4(row[k], vv[k], ww[k], (int)(unsigned)(c0 + p0 + k));
-                        fbuf[at] = (unsigned char)fl[k];
-                    }
-                    nsv += __popc(mk);
-                    cand[k] = false;   // (the item path below has nothing left to do)
-                }
-                __syncwarp();
-                for (int b0 = 0; b0 < nsv; b0 += 32) {
-                    const int at = b0 + lane;
-                    int4 e = make_int4(0, 0, 0, 0);
-                    bool kp = false;
-                    if (at < nsv) {
-                        e = buf[at];
-                        const unsigned f = fbuf[at];
-                        const int p = (f & 1u) ? giant : __ldca(sid + e.x);      // set(u), set(v)
-                        const int q = (f & 2u) ? giant : __ldca(sid + e.y);
-                        kp = p != q;                                             // the filter
-                        e.x = p;
-                        e.y = q;
-                        if (kp) {
-                            const long long key = make_key(e.z, (unsigned)e.w);  // L19
-                            rec(p, key);                                          // L20
-                            rec(q, key);                                          // L21
-                        }
-                    }
-                    const unsigned mk = __ballot_sync(kFull, kp);                 // L7
-                    if (kp) tst_cg<SOA>(out, cnt + __popc(mk & lt), e, P.wlcap);
-                    cnt += __popc(mk);
-                }
-                __syncwarp();
             }
 #pragma unroll
             for (int k = 0; k < kItems; ++k) {
