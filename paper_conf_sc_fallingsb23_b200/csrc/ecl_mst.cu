@@ -83,26 +83,6 @@ struct Timing {
 };
 static thread_local Timing g_timing;
 
-// Shared-memory carveout of the hot kernels: they use a few KB of shared
-// memory per CTA and lean on L1 for their cached loads (finds, guards, key
-// reads, bitmap bits), so ask for the smallest carveout that fits
-// (ECLMST_CARVEOUT=<percent> overrides, -1 leaves the driver's choice).
-static void set_carveout() {
-    int pct = cudaSharedmemCarveoutMaxL1;
-    if (const char* v = getenv("ECLMST_CARVEOUT")) pct = atoi(v);
-    if (pct < 0) return;
-    const void* fns[] = {
-        reinterpret_cast<const void*>(k_rounds<1, false, 0>), reinterpret_cast<const void*>(k_rounds<2, false, 0>),
-        reinterpret_cast<const void*>(k_populate<1, false, false>), reinterpret_cast<const void*>(k_populate<2, false, false>),
-        reinterpret_cast<const void*>(k_flatten<0>), reinterpret_cast<const void*>(k_flatten<1>),
-        reinterpret_cast<const void*>(k_flatten<2>), reinterpret_cast<const void*>(k_init),
-        reinterpret_cast<const void*>(k_dist_passA<true>), reinterpret_cast<const void*>(k_dist_passA<false>),
-        reinterpret_cast<const void*>(k_dist_reps1), reinterpret_cast<const void*>(k_dist_reps2),
-        reinterpret_cast<const void*>(k_dist_loop<1>), reinterpret_cast<const void*>(k_dist_loop<2>)};
-    for (const void* f : fns) cudaFuncSetAttribute(f, cudaFuncAttributePreferredSharedMemoryCarveout, pct);
-    cudaGetLastError();   // (a hint: never an error for the caller)
-}
-
 static int device_info(DevInfo* out) {
     int dev = 0;
     cudaError_t e = cudaGetDevice(&dev);
@@ -121,7 +101,6 @@ static int device_info(DevInfo* out) {
         if (!coop || occ < 1) return fail(ECL_MST_ERR_CUDA, "cooperative launch unsupported (coop=%d occ=%d)", coop, occ);
         g_dev[dev].sms = sms;
         g_dev[dev].occ = occ;
-        set_carveout();
     }
     *out = g_dev[dev];
     return ECL_MST_OK;
