@@ -520,6 +520,9 @@ __device__ __forceinline__ int split_threshold(const Params& P, const CSRC& S, l
                                      // scans: C2 2.261 -> 2.129 ms, C3 2.875 -> 2.810, C4 +-0, C1 +-0;
                                      // the first, one-id-per-lane scans had cost C2 +0.1 ms)
 #endif
+#ifndef ECL_RELABEL_FLAT
+#define ECL_RELABEL_FLAT 1
+#endif
 constexpr int kRlItems = 8;                     // ids per lane per step of a relabel scan
 constexpr int kRlStep = 32 * kRlItems;          // 256 ids per warp step
 __device__ __forceinline__ long long relabel(const Params& P, long long base, long long size, long long nbase,
@@ -590,6 +593,28 @@ __device__ __forceinline__ long long relabel(const Params& P, long long base, lo
         }
     }
     grid.sync();
+#if ECL_RELABEL_FLAT
+    // Flatten the closed level: every non-root id takes its root's label
+    // directly (~label, the root's own encoding), so the next pass A's finds
+    // from it -- and the flatten before phase 2 -- take one load.  Walks run
+    // concurrently; a walker meeting an id already rewritten stops there with
+    // the right label.  Four ids per thread in flight.
+    const long long gstride = (long long)G * kBlock;
+    for (long long x0 = base + (long long)b * kBlock + tid; x0 < end; x0 += 4 * gstride) {
+        int px[4];
+#pragma unroll
+        for (int a = 0; a < 4; ++a) px[a] = x0 + a * gstride < end ? __ldcg(P.parent + x0 + a * gstride) : -1;
+#pragma unroll
+        for (int a = 0; a < 4; ++a) {
+            if (px[a] >= 0) {
+                const long long x = x0 + a * gstride;
+                const int lab = find_label_from(P.parent, (int)x, px[a], false);
+                __stcg(P.parent + x, ~lab);
+            }
+        }
+    }
+    grid.sync();
+#endif
     return tot;
 }
 
