@@ -175,7 +175,7 @@ __global__ void __launch_bounds__(1024) k_qselect(Params P) {
 // ---------------------------------------------------------------------------
 // k_populate<PH>: one warp per 128-entry CSR chunk
 // ---------------------------------------------------------------------------
-template <int PH, bool SOA = false, bool BOTH = false>
+template <int PH, bool SOA = false, bool BOTH = false, int DEEP = -1>
 #ifndef ECL_DEEP_PH1
 #define ECL_DEEP_PH1 0
 #endif
@@ -255,7 +255,8 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
     };
     // deep: also prefetch the next chunk's row starts (phase 2, where the
     // bitmap / parent loads already lengthen each chunk's chain)
-    constexpr bool deep = PH == 1 ? ECL_DEEP_PH1 : ECL_DEEP_PH2;
+    // (DEEP >= 0: the host's choice; phase 1 of huge graphs takes it, see pop_kernel)
+    constexpr bool deep = DEEP >= 0 ? DEEP != 0 : (PH == 1 ? ECL_DEEP_PH1 : ECL_DEEP_PH2);
     auto bracket = [&](long long lc, int& r0, int& rl) {
         const long long c = P.shard + lc * P.nshards;
         r0 = __ldg(P.rowstart + c);
