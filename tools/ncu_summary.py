@@ -26,11 +26,9 @@ UNIT_SCALE = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12
 
 
 def stage_of(kernel_name):
-    k = kernel_name
-    for pat, st in (("k_init", "init"), ("k_populate<1>", "populate1"), ("k_populate<(int)1>", "populate1"),
-                    ("k_populate<2>", "populate2"), ("k_populate<(int)2>", "populate2"),
-                    ("k_rounds<1>", "rounds1"), ("k_rounds<(int)1>", "rounds1"),
-                    ("k_rounds<2>", "rounds2"), ("k_rounds<(int)2>", "rounds2"),
+    k = kernel_name.replace("(int)", "")
+    for pat, st in (("k_init", "init"), ("k_populate<1", "populate1"), ("k_populate<2", "populate2"),
+                    ("k_rounds<1", "rounds1"), ("k_rounds<2", "rounds2"), ("k_qhist", "init"), ("k_qselect", "init"),
                     ("k_flatten", "flatten"), ("k_giant", "flatten"), ("k_finalize", "finalize")):
         if pat in k:
             return st
