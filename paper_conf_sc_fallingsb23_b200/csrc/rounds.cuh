@@ -417,12 +417,15 @@ __device__ __forceinline__ void passB(const Params& P, const DS& D, const SRC& S
 // is far larger than L2 (n >= 2^25: every unguarded atomic on a random slot
 // is a DRAM read-modify-write, a guard miss only a read).  Measured: C5 and
 // C4 gain, C2/C3 lose with guards in every round.
+#ifndef ECL_GUARD_SLOTS
+#define ECL_GUARD_SLOTS (1 << 24)
+#endif
 __device__ __forceinline__ bool use_guard(const Params& P, long long live, long long winners, long long slots) {
     if (P.guards >= 0) return P.guards != 0;
     // (huge graphs, n >= 2^25: guard while the open level holds > 2^24 slots
     // (> 128 MB, beyond the L2); measured: C2's 24M-vertex level with guards
     // 1.68 -> 1.93 ms, C5's relabelled 19.7M-slot level without them +0.8 ms)
-    return live > 8 * winners || (P.n >= (1 << 25) && slots > (1 << 24));
+    return live > 8 * winners || (P.n >= (1 << 25) && slots > ECL_GUARD_SLOTS);
 }
 
 // ---------------------------------------------------------------------------

@@ -32,9 +32,12 @@ int main() {
     CUmulticastObjectProp prop = {};
     prop.numDevices = 1;
     prop.size = bytes;
-    prop.handleTypes = CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR;
-    size_t gran = 0;
+    prop.handleTypes = CU_MEM_HANDLE_TYPE_NONE;
+    size_t gran = 0, mgran = 0;
+    CK(cuMulticastGetGranularity(&mgran, &prop, CU_MULTICAST_GRANULARITY_MINIMUM));
     CK(cuMulticastGetGranularity(&gran, &prop, CU_MULTICAST_GRANULARITY_RECOMMENDED));
+    printf("granularity min %zu rec %zu\n", mgran, gran);
+    gran = mgran;
     prop.size = (bytes + gran - 1) / gran * gran;
     printf("granularity %zu size %zu\n", gran, prop.size);
     CUmemGenericAllocationHandle mch;
@@ -44,7 +47,7 @@ int main() {
     ap.type = CU_MEM_ALLOCATION_TYPE_PINNED;
     ap.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
     ap.location.id = 0;
-    ap.requestedHandleTypes = CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR;
+    ap.requestedHandleTypes = CU_MEM_HANDLE_TYPE_NONE;
     CUmemGenericAllocationHandle ph;
     CK(cuMemCreate(&ph, prop.size, &ap, 0));
     CK(cuMulticastBindMem(mch, 0, ph, 0, prop.size, 0));
