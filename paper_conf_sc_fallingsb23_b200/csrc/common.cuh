@@ -27,15 +27,6 @@ constexpr int kSplitSamples = 512;             // crowded-round threshold: about
 constexpr int kSplitSampleSlots = 1024;        // sample slots (max(1, 512 / G) per CTA, first CTAs)
 constexpr int kQBins = 2048;                   // exact-quantile radix select: 11 + 11 + 10 bits
 constexpr int kMaxLevels = 24;                 // relabel: contraction levels (level 0 = the vertices)
-// dynamic chunk scheduling of k_rounds' passes (rounds.cuh "work sharing"):
-// per-pass claim counters, per-CTA output counts (two parities), and every
-// CTA's populate-region chunk prefix
-constexpr int kMaxDynG = 512;                  // CTAs up to which the passes share work
-constexpr int kDynCtr = 2 * ECL_MST_MAX_ROUNDS + 8;
-constexpr int kDynCnt = kDynCtr;                        // [2][kMaxDynG] tuples per CTA arena, by round parity
-constexpr int kDynRtot = kDynCnt + 2 * kMaxDynG;          // [kMaxDynG] populate-region chunks per CTA
-constexpr int kDynRpre = kDynRtot + kMaxDynG;             // [kMaxDynG][kMaxRegionsPerCta + 1] their prefix
-constexpr int kDynInts = kDynRpre + kMaxDynG * (kMaxRegionsPerCta + 1);
 static_assert(kMaxGrid == ECL_MST_TRACE_CTAS, "trace layout");
 
 struct Internal {
@@ -65,8 +56,7 @@ struct Internal {
 };
 
 struct Layout {
-    size_t stats, internal, trace, rowstart, region, giant, samp, qhist, lvcnt, dyn, key, parent, setid, wl0, wl1,
-        total;
+    size_t stats, internal, trace, rowstart, region, giant, samp, qhist, lvcnt, key, parent, setid, wl0, wl1, total;
     long long wl_cap;                  // tuples per worklist buffer
 };
 
@@ -97,7 +87,6 @@ static inline Layout layout_for(int64_t n, int64_t M, int dup = 1) {
     L.samp = off;     off = align_up(off + sizeof(int) * (size_t)kSplitSampleSlots, 256);
     L.qhist = off;    off = align_up(off + sizeof(unsigned long long) * (size_t)kQBins, 256);
     L.lvcnt = off;    off = align_up(off + sizeof(int) * (size_t)kMaxGrid, 256);
-    L.dyn = off;      off = align_up(off + sizeof(int) * (size_t)kDynInts, 256);
     // key / parent: 2n slots, the vertices plus the contraction levels (Internal)
     L.key = off;      off = align_up(off + sizeof(long long) * (size_t)(2 * n), 256);
     L.parent = off;   off = align_up(off + sizeof(int) * (size_t)(2 * n), 256);
@@ -147,7 +136,6 @@ struct Params {
     int* samp;                        // crowded-round weight samples (kSplitSampleSlots)
     unsigned long long* qhist;        // exact-quantile histogram (kQBins)
     int relabel;                      // -1 auto, 0 off, 1 whenever the sets at least halved (opts.relabel)
-    int* dyn;                         // work sharing state (kDynInts; null: static arenas only)
     int* lvcnt;                       // per-CTA root counts of a relabel (kMaxGrid)
     int* setid;                       // set of every vertex after phase 1 (k_flatten), read by populate 2
     long long wlcap;                  // tuples per worklist buffer (plane stride of opts.tuple_layout 1)

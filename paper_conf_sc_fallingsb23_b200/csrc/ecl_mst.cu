@@ -353,10 +353,6 @@ static int run_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t
     P.relabel = (o.flatten && (long long)n <= (1LL << 30)) ? (o.relabel < 0 ? -1 : (o.relabel ? 1 : 0)) : 0;
     P.lvcnt = reinterpret_cast<int*>(ws + L.lvcnt);
     P.setid = reinterpret_cast<int*>(ws + L.setid);
-#ifndef ECL_DYN
-#define ECL_DYN 1
-#endif
-    P.dyn = ECL_DYN ? reinterpret_cast<int*>(ws + L.dyn) : nullptr;   // work sharing in k_rounds' passes
     P.wlcap = L.wl_cap;
     P.both = o.both_directions ? 1 : 0;
     P.drive = o.drive;
@@ -981,7 +977,6 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
         P.qhist = reinterpret_cast<unsigned long long*>(ws + L.qhist);
         P.relabel = 0;   // (the replicated union-find stays on vertex ids)
         P.lvcnt = nullptr;
-        P.dyn = nullptr;
         P.setid = reinterpret_cast<int*>(ws + L.setid);
         P.wlcap = L.wl_cap;
         P.both = 0;

@@ -91,8 +91,6 @@ __global__ void __launch_bounds__(256) k_init(Params P) {
         }
         if (P.threshold_mode == 2)
             for (int i = tid; i < kQBins; i += blockDim.x) P.qhist[i] = 0;
-        if (P.dyn)   // work sharing: every pass's claim counter starts at 0
-            for (int i = tid; i < kDynCtr; i += blockDim.x) P.dyn[i] = 0;
     }
     if (err) atomicExch(&P.st->status, ECL_MST_ERR_INPUT);
 }

@@ -112,7 +112,6 @@ __global__ void __launch_bounds__(256) k_giant(Params P) {
 template <bool SOA_ = false>
 struct CompactSrcT {
     static constexpr bool SOA = SOA_;
-    static constexpr bool DYN = false;
     const int4* base;
     int cnt;
     int nloc;
@@ -126,7 +125,6 @@ using CompactSrc = CompactSrcT<false>;
 template <bool SOA_ = false>
 struct RegionSrcT {
     static constexpr bool SOA = SOA_;
-    static constexpr bool DYN = false;
     const int* s_pre;   // shared memory: chunk prefix per region (nreg + 1)
     const int* s_rcnt;  // shared memory: tuples per region
     int nreg;
@@ -151,7 +149,6 @@ using RegionSrc = RegionSrcT<false>;
 template <bool SOA_ = false>
 struct GlobalSrcT {
     static constexpr bool SOA = SOA_;
-    static constexpr bool DYN = false;
     const int4* base;
     long long cnt;
     int nloc;
@@ -170,103 +167,6 @@ __device__ __forceinline__ GlobalSrcT<SOA> global_src(const int4* base, long lon
     const long long nch = (cnt + kChunk - 1) / kChunk;
     S.nloc = blockIdx.x < nch ? (int)((nch - blockIdx.x + gridDim.x - 1) / gridDim.x) : 0;
     return S;
-}
-
-// ---------------------------------------------------------------------------
-// Work sharing.  A CTA's own arena is a static share of a pass, and CTAs
-// finish at different times (C5 round 0 pass B: first CTA after 2.5 ms, last
-// after 4.3 ms) while the grid barrier waits for the last.  With a DynSrcT
-// every warp claims its next chunk from one counter per pass, over the
-// concatenation of all CTAs' arenas (REGION: of all CTAs' populate regions);
-// pass A still appends to its own CTA's arena, and claims only while that
-// arena has room, so nothing downstream changes.
-// ---------------------------------------------------------------------------
-template <bool SOA_, bool REGION>
-struct DynSrcT {
-    static constexpr bool SOA = SOA_;
-    static constexpr bool DYN = true;
-    const int* s_cpre;      // shared: chunk prefix over the CTAs (G + 1 entries)
-    const int* cnt;         // compact: tuples per CTA arena
-    const int4* base;       // compact: the buffer
-    int G;
-    int nloc;               // chunks of the pass
-    int* ctr;               // the pass's claim counter
-    __device__ __forceinline__ const int4* get(const Params& P, int k, int& count) const {
-        int lo = 0, hi = G;   // the CTA whose arena holds chunk k
-        while (hi - lo > 1) {
-            const int mid = (lo + hi) >> 1;
-            if (s_cpre[mid] <= k) lo = mid;
-            else hi = mid;
-        }
-        const int j = k - s_cpre[lo];
-        if (!REGION) {
-            count = min(kChunk, __ldcg(cnt + lo) - j * kChunk);
-            return tadd<SOA>(base, (long long)lo * P.cap + (long long)j * kChunk);
-        }
-        // CTA lo's regions lo, lo + G, ...: their chunk prefix (k_rounds start)
-        const int* rp = P.dyn + kDynRpre + lo * (kMaxRegionsPerCta + 1);
-        int a = 0, b = (P.W - lo + P.G - 1) / P.G;
-        while (b - a > 1) {
-            const int mid = (a + b) >> 1;
-            if (__ldg(rp + mid) <= j) a = mid;
-            else b = mid;
-        }
-        const int off = j - __ldg(rp + a);
-        const int w = lo + a * P.G;
-        count = min(kChunk, __ldg(&P.region[w].x) - off * kChunk);
-        return tadd<SOA>(P.wl0, (long long)w * P.rcap + (long long)off * kChunk);
-    }
-};
-
-// the shared chunk prefix of a dynamic pass from per-CTA counts (tuples, or
-// chunks when CHUNKS): every thread of the CTA calls it; returns the total
-template <bool CHUNKS>
-__device__ __forceinline__ int dyn_prefix(const int* cnt, int G, int* s_cpre, int* s_tmp) {
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    int v = 0;
-    if (tid < G) {
-        v = __ldcg(cnt + tid);
-        if (!CHUNKS) v = (v + kChunk - 1) / kChunk;
-    }
-    int incl = v;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-        const int y = __shfl_up_sync(kFull, incl, o);
-        if (lane >= o) incl += y;
-    }
-    if (lane == 31) s_tmp[warp] = incl;
-    __syncthreads();
-    int wbase = 0;
-    for (int w = 0; w < warp; ++w) wbase += s_tmp[w];
-    if (tid < G) s_cpre[tid + 1] = wbase + incl;
-    if (tid == 0) s_cpre[0] = 0;
-    __syncthreads();
-    const int tot = s_cpre[G];
-    __syncthreads();
-    return tot;
-}
-
-// visit the chunks of S: static sources give warp w the chunks w, w + kWarps,
-// ... of the CTA's own arena; dynamic ones hand out chunks from the pass's
-// counter (one atomic per warp and chunk) while the CTA's claimed tuples stay
-// within `budget` (pass A's output arena)
-template <class SRC, class F>
-__device__ __forceinline__ void for_chunks(const SRC& S, bool reverse, long long budget, int* s_claim, F&& body) {
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    if constexpr (SRC::DYN) {
-        for (;;) {
-            int k = INT_MAX;
-            if (lane == 0 && *reinterpret_cast<volatile int*>(s_claim) + (long long)kWarps * kChunk <= budget) {
-                k = atomicAdd(S.ctr, 1);
-                if (k < S.nloc) atomicAdd(s_claim, kChunk);
-            }
-            k = __shfl_sync(kFull, k, 0);
-            if (k >= S.nloc) break;
-            body(reverse ? S.nloc - 1 - k : k);
-        }
-    } else {
-        for (int kk = warp; kk < S.nloc; kk += kWarps) body(reverse ? S.nloc - 1 - kk : kk);
-    }
 }
 
 template <class T>
@@ -348,10 +248,10 @@ __device__ __forceinline__ RegionSrcT<SOA> region_src(const Params& P, int b, in
 template <bool SPLIT = false, bool MAP = false, class SRC>
 __device__ __forceinline__ void passA(const Params& P, const DS& D, const SRC& S, int4* __restrict__ out,
                                       int* s_out, bool guard, int T = INT_MAX, int4* out_end = nullptr,
-                                      int* s_def = nullptr, long long budget = LLONG_MAX, int* s_claim = nullptr) {
-    const int lane = threadIdx.x & 31;
+                                      int* s_def = nullptr) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const bool halving = P.halving != 0;
-    for_chunks(S, false, budget, s_claim, [&](int k) {
+    for (int k = warp; k < S.nloc; k += kWarps) {
         int count;
         const int4* __restrict__ in = S.get(P, k, count);
         int4 t[kItems];
@@ -400,7 +300,7 @@ __device__ __forceinline__ void passA(const Params& P, const DS& D, const SRC& S
             }
         }
         warp_emit<SRC::SOA>(t, keep, out, s_out, P.wlcap);                // L18
-    });
+    }
 }
 
 // opts.drive 2, "Vertex-Centric": pass A as one thread per vertex
@@ -447,13 +347,13 @@ __device__ __forceinline__ void passA_vc(const Params& P, const DS& D, unsigned 
 // level's best-edge slots, so the winners leave them as they are (k_rounds
 // refills them should the relabel not happen after all).
 template <bool NORESET = false, class SRC>
-__device__ __forceinline__ void passB(const Params& P, const DS& D, const SRC& S, long long* acc,
-                                      int* s_claim = nullptr) {
-    const int lane = threadIdx.x & 31;
-    // (ECL_B_REVERSE: walk the chunks back to front, so pass B starts on the
-    // tuples the last pass wrote most recently, still in L2, and the next
-    // pass A, walking front to back, starts on the ones pass B read last)
-    for_chunks(S, ECL_B_REVERSE != 0, LLONG_MAX, s_claim, [&](int k) {
+__device__ __forceinline__ void passB(const Params& P, const DS& D, const SRC& S, long long* acc) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    for (int kk = warp; kk < S.nloc; kk += kWarps) {
+        // (ECL_B_REVERSE: walk the chunks back to front, so pass B starts on the
+        // tuples the last pass wrote most recently, still in L2, and the next
+        // pass A, walking front to back, starts on the ones pass B read last)
+        const int k = ECL_B_REVERSE ? S.nloc - 1 - kk : kk;
         int count;
         const int4* __restrict__ in = S.get(P, k, count);
         int4 t[kItems];
@@ -507,7 +407,7 @@ __device__ __forceinline__ void passB(const Params& P, const DS& D, const SRC& S
                 acc[1] += ccnt;
             }
         }
-    });
+    }
 }
 
 // guard policy for pass A.  "auto" guards when edges crowd onto few
@@ -754,14 +654,6 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
     // the populate output of this CTA: regions w = b, b + G, ... (region mode)
     const RegionSrcT<SOA> R = region_src<SOA>(P, b, s_pre, s_rcnt, s_red, &st->live[g], PH == 1);
     if (b0 && tid == 0 && PH == 2) st->phase2_round = g;
-    // work sharing (see DynSrcT): every CTA publishes its regions' chunk prefix
-    const bool dyn = P.dyn != nullptr && P.G <= kMaxDynG && DRIVE == 0;
-    if (dyn) {
-        for (int k = tid; k <= R.nreg; k += kBlock) P.dyn[kDynRpre + b * (kMaxRegionsPerCta + 1) + k] = s_pre[k];
-        if (tid == 0) P.dyn[kDynRtot + b] = R.nloc;
-    }
-    __shared__ int s_cpre[kMaxDynG + 1];
-    __shared__ int s_claim;
     trace_cta(P, 4 + 2 * g);
     grid.sync();
     __shared__ long long s_acc[kWarps][2];   // per warp: MSF weight, MSF edges (pass B)
@@ -799,37 +691,14 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
                (P.relabel > 0 || (lv_size >= ECL_RELABEL_MIN && 4 * L >= lv_size &&
                                   (s_lev > 0 || lv_size >= ECL_RELABEL_FIRST)));
     };
-    // the dynamic view of the pass's input: all CTAs' populate regions (first
-    // round) or all CTAs' arenas of buffer `buf` (counts of parity `par`)
-    auto dyn_src = [&](const auto& S, int pass_id, int par, int buf) {
-        constexpr bool REG = !is_compact_src<std::decay_t<decltype(S)>>::value;
-        DynSrcT<SOA, REG> X;
-        const int* cnt = REG ? P.dyn + kDynRtot : P.dyn + kDynCnt + par * kMaxDynG;
-        X.nloc = dyn_prefix<REG>(cnt, P.G, s_cpre, s_wc);
-        X.s_cpre = s_cpre;
-        X.cnt = cnt;
-        X.base = buf ? P.wl1 : P.wl0;
-        X.G = P.G;
-        X.ctr = P.dyn + pass_id;
-        if (tid == 0) s_claim = 0;
-        __syncthreads();
-        return X;
-    };
     auto round = [&](const auto& S) {
         const long long w0 = acc[1];
         const bool noreset = may_relabel();
         // (both_directions: an edge's two copies must see the same slots, so
         // no copy resets them in pass B; the paper's separate reset kernel,
         // L34-37, follows instead)
-        if (dyn) {
-            const auto X = dyn_src(S, 2 * g, g & 1, cur);
-            if (noreset || P.both) passB<true>(P, D, X, acc, &s_claim);
-            else passB(P, D, X, acc, &s_claim);
-        } else if (noreset || P.both) {
-            passB<true>(P, D, S, acc);
-        } else {
-            passB(P, D, S, acc);
-        }
+        if (noreset || P.both) passB<true>(P, D, S, acc);
+        else passB(P, D, S, acc);
         const long long d = acc[1] - w0;
         if (lane == 0 && d) atomicAdd(reinterpret_cast<unsigned long long*>(&st->winners[g]), (unsigned long long)d);
         if (tid == 0) s_out = s_def = 0;
@@ -902,16 +771,6 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
             passA_vc<PH, SOA>(P, D, vcnt, guard);
         } else if constexpr (topo) {
             passA(P, D, R, wl[1], &s_out, guard);
-        } else if (dyn && hb < 0 && (long long)P.G * (P.cap - kWarps * kChunk - kChunk) >= L) {
-            // (every CTA claims while its own output arena has room; the
-            // arenas together hold the whole input, so every chunk is taken)
-            const auto X = dyn_src(S, 2 * g + 1, (g - 1) & 1, cur);
-            if (T != INT_MAX)
-                passA<true>(P, D, X, wl[cur ^ 1], &s_out, guard, T, tadd<SOA>(wl[cur ^ 1], P.cap), &s_def, P.cap,
-                            &s_claim);
-            else if (mapped) passA<false, true>(P, D, X, wl[cur ^ 1], &s_out, guard, INT_MAX, nullptr, nullptr, P.cap,
-                                                &s_claim);
-            else passA(P, D, X, wl[cur ^ 1], &s_out, guard, INT_MAX, nullptr, nullptr, P.cap, &s_claim);
         } else if (T != INT_MAX)
             passA<true>(P, D, S, wl[cur ^ 1], &s_out, guard, T, tadd<SOA>(wl[cur ^ 1], P.cap), &s_def);
         else if (mapped) passA<false, true>(P, D, S, wl[cur ^ 1], &s_out, guard);
@@ -919,7 +778,6 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
         cur = topo ? 1 : cur ^ 1;
         __syncthreads();
         C = compact_src<SOA>(wl[cur], s_out);
-        if (dyn && tid == 0) P.dyn[kDynCnt + (g & 1) * kMaxDynG + b] = s_out;   // this pass's arenas, by parity
         if (T != INT_MAX) {
             hb = cur;
             hcnt = s_def;
@@ -956,7 +814,6 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
         cur = ob;
         __syncthreads();
         C = compact_src<SOA>(wl[cur], s_out);
-        if (dyn && tid == 0) P.dyn[kDynCnt + (g & 1) * kMaxDynG + b] = s_out;
         if (tid == 0 && C.cnt) atomicAdd(reinterpret_cast<unsigned long long*>(&st->live[g]), (unsigned long long)C.cnt);
         trace_cta(P, 4 + 2 * g);
         grid.sync();
