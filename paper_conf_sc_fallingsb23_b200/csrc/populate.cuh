@@ -185,6 +185,9 @@ template <int PH, bool SOA = false, bool BOTH = false, int DEEP = -1>
 #ifndef ECL_GIANT_MIN_N
 #define ECL_GIANT_MIN_N (32LL << 20)   // parent[] larger than ~half the L2
 #endif
+#ifndef ECL_EARLY_VBITS
+#define ECL_EARLY_VBITS 1
+#endif
 #ifndef ECL_P2_GUARD_COLD
 #define ECL_P2_GUARD_COLD 0   // phase-2 populate: guard the atomicMin of slots other than the giant's
                               // (off: C4 populate2 2.60 -> 2.40 ms, C5 11.8 -> 11.4 ms)
@@ -390,6 +393,11 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
                     if (p0 + k < len) P.in_mst[c0 + p0 + k] = 0;
             }
         }
+#if ECL_EARLY_VBITS
+        // the next chunk's far-end bits, issued half a chunk earlier than at
+        // the end of this one (its entries have arrived by now)
+        if (PH == 2 && lcn < lend) nvb = vbits(nv, nw, nr0);
+#endif
         bool cand[kItems];
 #pragma unroll
         for (int k = 0; k < kItems; ++k) {
@@ -478,7 +486,9 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
             }
         }
     }
+#if !ECL_EARLY_VBITS
     if (PH == 2 && nxt(lc) < lend) nvb = vbits(nv, nw, nr0);   // next chunk's far-end bits
+#endif
     // L7: append the chunk's tuples to the warp's region (both_directions:
     // then their mirror copies <q, p, w, id>)
     for (int copy = 0; copy < 1 + BOTH; ++copy) {
