@@ -85,7 +85,7 @@ __global__ void __launch_bounds__(256) k_dist_reps1(Params P, const int* R, long
 // tuple-centric pass B, so the partition after each round is the same.
 // keep[i]: x stays a root with a live edge (the next round's R).
 __global__ void __launch_bounds__(256) k_dist_reps2(Params P, const int* R, long long nR, const long long* buf,
-                                                    unsigned char* keep, int g, long long* hbuf = nullptr) {
+                                                    unsigned char* keep, int g) {
     const long long stride = (long long)gridDim.x * blockDim.x;
     long long wsum = 0, wcnt = 0;
     unsigned long long found = 0;   // sets with a finite key (0: the phase is done)
@@ -97,18 +97,9 @@ __global__ void __launch_bounds__(256) k_dist_reps2(Params P, const int* R, long
             continue;
         }
         ++found;
-        int q;
-        bool mutual;
-        if (hbuf) {   // from the tuple-centric pass B (k_dist_passB), reduced over the ranks
-            const long long hv = hbuf[i];
-            hbuf[i] = 0;   // (ready for the next round)
-            q = (int)(hv & 0xffffffffll);
-            mutual = ((hv >> 32) & 1) != 0;
-        } else {
-            const int t = P.tgt[i];
-            q = t & 0x7fffffff;
-            mutual = t < 0;
-        }
+        const int t = P.tgt[i];
+        const int q = t & 0x7fffffff;
+        const bool mutual = t < 0;
         if (!mutual || (int)x > q) P.parent[x] = q;
         if (!mutual || (int)x < q) {
             P.in_mst[(unsigned)(kx & 0xffffffffll)] = 1;
@@ -171,7 +162,7 @@ __global__ void __launch_bounds__(kCompactBlock) k_dist_compact(const int* R, lo
                                                                 const int* bcnt, int* Rnext, long long* nnext,
                                                                 unsigned long long* reps,
                                                                 volatile long long* host_out,
-                                                                const DistSplit* dsp, int* pos = nullptr) {
+                                                                const DistSplit* dsp) {
     __shared__ int s_base, s_w[kCompactBlock / 32];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     {   // this block's offset: the counts of the blocks before it (block-wide sum)
@@ -217,53 +208,8 @@ __global__ void __launch_bounds__(kCompactBlock) k_dist_compact(const int* R, lo
         const long long i = i0 + lane;
         const bool k = i < whi && keep[i];
         const unsigned m = __ballot_sync(kFull, k);
-        if (k) {
-            const int x = (int)set_of(R, i);
-            Rnext[base + __popc(m & lt)] = x;
-            if (pos) pos[x] = base + __popc(m & lt);   // (k_dist_passB: set -> its place in the list)
-        }
+        if (k) Rnext[base + __popc(m & lt)] = (int)set_of(R, i);
         base += __popc(m);
-    }
-}
-
-// Tuple-centric rep pass 1 (replaces k_dist_reps1's edge-id lookups): after
-// the key exchange, every rank walks its own tuples; a tuple whose id is the
-// reduced key of its set p (or q) is that set's lightest edge, and it knows
-// the other end directly.  It publishes {q, mutual} at p's place in the root
-// list (and {p, mutual} at q's), as 1 << 40 | mutual << 32 | other, so an
-// allreduce(max) over the ranks gives every rank the hook of every set (each
-// edge lives on exactly one rank; 0 = no hook from here).
-template <bool FIRST>
-__global__ void __launch_bounds__(kBlock, 2) k_dist_passB(Params P, const long long* red, const int* pos,
-                                                         long long* hbuf, int cur) {
-    __shared__ long long s_red[3][kWarps];
-    __shared__ int s_pre[kMaxRegionsPerCta + 1];
-    __shared__ int s_rcnt[kMaxRegionsPerCta];
-    const int lane = threadIdx.x & 31;
-    const int b = blockIdx.x;
-    if (FIRST && !input_ok(P)) return;
-    auto visit = [&](const auto& S) {
-        for (int k = threadIdx.x >> 5; k < S.nloc; k += kWarps) {
-            int count;
-            const int4* in = S.get(P, k, count);
-#pragma unroll
-            for (int i0 = 0; i0 < kItems; ++i0) {
-                const int idx = i0 * 32 + lane;
-                if (idx >= count) continue;
-                const int4 t = __ldcg(in + idx);
-                const unsigned kp = __ldcg(reinterpret_cast<const unsigned*>(red + t.x));
-                const unsigned kq = __ldcg(reinterpret_cast<const unsigned*>(red + t.y));
-                const bool wp = kp == (unsigned)t.w, wq = kq == (unsigned)t.w;
-                const long long mut = (wp && wq) ? (1LL << 32) : 0;
-                if (wp) hbuf[pos ? pos[t.x] : t.x] = (1LL << 40) | mut | (unsigned)t.y;
-                if (wq) hbuf[pos ? pos[t.y] : t.y] = (1LL << 40) | mut | (unsigned)t.x;
-            }
-        }
-    };
-    if (FIRST) {
-        visit(region_src(P, b, s_pre, s_rcnt, s_red, nullptr, false));
-    } else {
-        visit(compact_src((cur ? P.wl1 : P.wl0) + (long long)b * P.cap, P.acnt[b]));
     }
 }
 

@@ -701,7 +701,7 @@ struct NcclApi {
     int (*commDestroy)(NcclComm) = nullptr;
     const char* (*getErrorString)(int) = nullptr;
 };
-constexpr int kNcclInt32 = 2, kNcclInt64 = 4, kNcclSum = 0, kNcclMax = 2, kNcclMin = 3;
+constexpr int kNcclInt32 = 2, kNcclInt64 = 4, kNcclSum = 0, kNcclMin = 3;
 static NcclApi g_nccl;
 static std::mutex g_nccl_mu;
 
@@ -745,7 +745,7 @@ static void release(DistHandle* h) {
 
 struct DistLayout {
     size_t stats, internal, rowstart, parent, tgt, keyptrs, rl0, rl1, rbuf, keep, bcnt, dsplit, giant, qhist, setid,
-        sps, found, hbuf, pos, shard0, shard_bytes, total;
+        sps, found, shard0, shard_bytes, total;
     size_t region, acnt, hcnt, key, wl0, wl1;   // offsets inside one shard block
     long long wl_cap, nlocal_max;
 };
@@ -774,8 +774,6 @@ static inline DistLayout dist_layout(int64_t n, int64_t M, int S, int world) {
     L.qhist = off;    off = align_up(off + sizeof(unsigned long long) * (size_t)kQBins, 256);
     L.setid = off;    off = align_up(off + sizeof(int) * (size_t)n, 256);
     L.sps = off;      off = align_up(off + sizeof(Params) * (size_t)S, 256);   // dist_loop: the shards' Params
-    L.hbuf = off;     off = align_up(off + sizeof(long long) * (size_t)n, 256);   // hooks by root-list place
-    L.pos = off;      off = align_up(off + sizeof(int) * (size_t)n, 256);         // set -> root-list place
     L.found = off;    off = align_up(off + 2 * sizeof(unsigned long long), 256);
     size_t so = 0;
     L.region = so; so = align_up(so + sizeof(int4) * (size_t)kMaxPopWarps, 256);
@@ -1021,7 +1019,6 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
     if (e == cudaSuccess) e = cudaMemsetAsync(in, 0, sizeof(Internal), s);   // (reps: zeroed again by each k_dist_compact)
     if (e == cudaSuccess) e = cudaMemsetAsync(&dsp->hb, 0xFF, sizeof(int), s);    // hb = -1: nothing deferred
     if (e == cudaSuccess) e = cudaMemsetAsync(in_mst_out, 0, (size_t)M, s);   // every rank returns the full mask
-    if (e == cudaSuccess) e = cudaMemsetAsync(ws + L.hbuf, 0, sizeof(long long) * (size_t)n, s);   // (k_dist_reps2 re-zeroes)
     if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "memset: %s", cudaGetErrorString(e));
     k_init<<<vblocks, 256, 0, s>>>(P0);
     if ((rc = check("k_init"))) return rc;
@@ -1030,7 +1027,6 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
     int g = 0;
     int* const rlist[2] = {reinterpret_cast<int*>(ws + L.rl0), reinterpret_cast<int*>(ws + L.rl1)};
     unsigned char* const rkeep = reinterpret_cast<unsigned char*>(ws + L.keep);
-    int* const rpos = reinterpret_cast<int*>(ws + L.pos);   // set -> place in the root list (k_dist_passB)
     int* const rcnt = reinterpret_cast<int*>(ws + L.bcnt);
     long long phase2_roots = 0;
     // the current roots into `out` (count: h_map[1] after the next sync)
@@ -1038,8 +1034,8 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
         const unsigned cb = (unsigned)std::max<long long>(1, std::min<long long>(ceil_div(n, 4096), kCompactGridMax));
         k_dist_root_keep<<<vblocks, 256, 0, s>>>(P0, rkeep);
         k_dist_count<<<cb, kCompactBlock, 0, s>>>(n, rkeep, rcnt);
-        k_dist_compact<<<cb, kCompactBlock, 0, s>>>(nullptr, n, rkeep, rcnt, out, &in->nroots, &in->reps, h->d_map, nullptr,
-                                                    rpos);
+        k_dist_compact<<<cb, kCompactBlock, 0, s>>>(nullptr, n, rkeep, rcnt, out, &in->nroots, &in->reps, h->d_map,
+                                                    nullptr);
     };
     if (dloop) {   // ---- device-initiated rounds: one persistent kernel per phase ----
         Params* d_sps = reinterpret_cast<Params*>(ws + L.sps);
@@ -1163,24 +1159,10 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
                 if ((rc = allreduce(rbuf, (size_t)nR + (split ? kSplitExt : 0), kNcclMin))) return rc;
                 k_dist_scatter<<<rblocks, 256, 0, s>>>(P0, R, nR, rbuf);
             }
-#ifndef ECL_DIST_PASSB
-#define ECL_DIST_PASSB 1
-#endif
-            // rep pass 1: every set's hook.  Default: the tuple-centric pass
-            // over each shard's own tuples (k_dist_passB; the set's lightest
-            // edge is some rank's tuple and knows the other end), reduced
-            // over the ranks by an allreduce(max).  Else: the edge-id lookups
-            // of k_dist_reps1 (row search and finds), split over the ranks
-            // (and over the virtual shards, which share tgt[]), then tgt[] is
-            // allgathered.  Pass 2 is replicated.
-            long long* const hbuf = ECL_DIST_PASSB ? reinterpret_cast<long long*>(ws + L.hbuf) : nullptr;
-            if (hbuf && nR > 0) {
-                for (int k = 0; k < S; ++k) {
-                    if (first) k_dist_passB<true><<<sp[k].G, kBlock, 0, s>>>(sp[k], P0.key, R ? rpos : nullptr, hbuf, cur);
-                    else k_dist_passB<false><<<sp[k].G, kBlock, 0, s>>>(sp[k], P0.key, R ? rpos : nullptr, hbuf, cur);
-                }
-                if ((rc = allreduce(hbuf, (size_t)nR, kNcclMax))) return rc;
-            } else if (nR > 0) {
+            // rep pass 1 -- the row search and finds, the costly part -- is
+            // split over the ranks (and over the virtual shards, which share
+            // tgt[]), then tgt[] is allgathered; pass 2 is replicated
+            if (nR > 0) {
                 const long long parts = world > 1 ? world : S;
                 const long long slice = ceil_div(nR, parts);
                 const unsigned sblocks = (unsigned)std::max<long long>(1, std::min<long long>(ceil_div(slice, 256), (long long)di.sms * 8));
@@ -1192,10 +1174,10 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
                     if (r) return fail(ECL_MST_ERR_CUDA, "ncclAllGather: %s", g_nccl.getErrorString ? g_nccl.getErrorString(r) : "?");
                 }
             }
-            k_dist_reps2<<<rblocks, 256, 0, s>>>(P0, R, nR, xbuf, keep, g, hbuf);
+            k_dist_reps2<<<rblocks, 256, 0, s>>>(P0, R, nR, xbuf, keep, g);
             k_dist_count<<<cblocks, kCompactBlock, 0, s>>>(nR, keep, bcnt);
             k_dist_compact<<<cblocks, kCompactBlock, 0, s>>>(R, nR, keep, bcnt, rl[rb], &in->nroots, &in->reps, h->d_map,
-                                                             split_on ? dsp : nullptr, rpos);
+                                                             split_on ? dsp : nullptr);
             e = cudaEventRecord(h->ev, s);
             if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "event: %s", cudaGetErrorString(e));
             const bool can_continue = g + 1 < ECL_MST_MAX_ROUNDS;
