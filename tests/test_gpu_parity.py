@@ -115,6 +115,10 @@ def test_config_small(eclmst, name):
     dict(relabel=1), dict(relabel=0), dict(relabel=1, refilter=1), dict(relabel=1, giant_bitmap=1),
     dict(relabel=1, max_ctas=3), dict(relabel=1, path_halving=0), dict(relabel=1, filter=0),
     dict(relabel=1, refilter=1, filter=1, filter_c=1, giant_bitmap=1), dict(relabel=1, atomic_guards=1),
+    # contraction inside phase 2 (threshold 0: nearly every edge is heavy) and with no phase 2 at all
+    dict(relabel=1, filter=1, threshold_mode=1, threshold=0), dict(relabel=1, filter=1, threshold_mode=1,
+                                                                   threshold=(1 << 31) - 1),
+    dict(relabel=1, max_ctas=1), dict(relabel=1, threshold_mode=2, giant_bitmap=1),
     # the Table-5 de-optimisations, one at a time and all together
     dict(populate_mode=1), dict(both_directions=1), dict(tuple_layout=1), dict(drive=1), dict(drive=2),
     dict(populate_mode=1, both_directions=1, tuple_layout=1, drive=2, atomic_guards=0, filter=0, path_halving=0,
@@ -486,3 +490,20 @@ def test_ids_above_2_31():
     assert got.numel() == n - 1
     assert torch.equal(got, torch.sort(expect_ids).values)
     assert int(got.max()) > (1 << 31)      # ids beyond the signed range were marked
+
+
+@pytest.mark.parametrize("seed", range(8))
+def test_contraction_levels(eclmst, seed):
+    """Forced contraction on graphs that need many rounds (long paths of
+    tie-heavy cycles joined into a ring, heavy-tailed degrees): many closed
+    levels in both phases, the flatten walking all of them, stats consistent."""
+    kinds = ["ties", "two", "uniform", "full"]
+    n = 2000 + 700 * seed
+    g = G.random_small(n, 3 * n, seed=7000 + seed, weights=kinds[seed % 4], multi=True, self_loops=True)
+    for opts in (dict(relabel=1), dict(relabel=1, filter=1, filter_c=1), dict(relabel=1, filter=1, filter_c=2,
+                                                                            refilter=1)):
+        st = assert_parity(eclmst, g, **opts)
+        check_round_bound(g, st)
+        assert st["relabels"] >= 1, opts
+    st = assert_parity(eclmst, G.path_graph(50_000), relabel=1)     # monotone path: one hook chain
+    assert st["relabels"] >= 1
