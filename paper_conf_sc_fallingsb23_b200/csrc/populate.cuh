@@ -426,12 +426,14 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
             for (int k = 0; k < kItems; ++k) {
                 const int wi = (row[k] >> 5) - (r0 >> 5);
                 const unsigned wd = __shfl_sync(kFull, rw, wi & 31);
-                rbit[k] = (deep && wi < 32) ? (wd >> (row[k] & 31)) & 1u : 2u;
+                // (a row beyond the lanes' 32 words -- a chunk spanning over
+                // 1024 rows -- counts as outside the set: its edges then
+                // take the setid path, which decides the same)
+                rbit[k] = (deep && wi < 32) ? (wd >> (row[k] & 31)) & 1u : 0u;
             }
 #pragma unroll
             for (int k = 0; k < kItems; ++k) {
-                if (cand[k] && giant >= 0 && ((vb >> k) & 1u) &&
-                    (rbit[k] == 2u ? (__ldg(P.giant_bits + (row[k] >> 5)) >> (row[k] & 31)) & 1u : rbit[k])) {
+                if (cand[k] && giant >= 0 && ((vb >> k) & 1u) && rbit[k]) {
                     pk[k] = qk[k] = giant;                    // both ends in the largest set: filtered
                 } else if (cand[k]) {
                     pk[k] = (k > 0 && cand[k - 1] && row[k] == row[k - 1]) ? -1 : __ldca(sid + row[k]);
