@@ -66,18 +66,33 @@ __global__ void __launch_bounds__(256) k_dist_scatter(Params P, const int* R, lo
 __global__ void __launch_bounds__(256) k_dist_reps1(Params P, const int* R, long long lo, long long hi,
                                                     const long long* buf) {
     const long long stride = (long long)gridDim.x * blockDim.x;
-    for (long long i = lo + (long long)blockIdx.x * blockDim.x + threadIdx.x; i < hi; i += stride) {
-        const long long kx = buf[i];
-        if (kx == kInf) continue;
-        const long long x = set_of(R, i);
-        const unsigned j = (unsigned)(kx & 0xffffffffll);
-        const int u = row_of_entry(P, (long long)j);
-        const int v = __ldg(P.nlist + j);
-        const DS D = ds_of(P);
-        const int pu = find_root(D, u, false), pv = find_root(D, v, false);
-        const int q = (pu == (int)x) ? pv : pu;
-        const bool mutual = P.key[q] == kx;
-        P.tgt[i] = q | (mutual ? (int)0x80000000 : 0);
+    const DS D = ds_of(P);
+    // four sets per thread in flight: each is a chain of dependent loads
+    // (row search, nlist, two finds, the other end's key)
+    for (long long i0 = lo + (long long)blockIdx.x * blockDim.x + threadIdx.x; i0 < hi; i0 += 4 * stride) {
+        long long kx[4];
+        int u[4], v[4];
+#pragma unroll
+        for (int a = 0; a < 4; ++a) {
+            const long long i = i0 + a * stride;
+            kx[a] = i < hi ? buf[i] : kInf;
+        }
+#pragma unroll
+        for (int a = 0; a < 4; ++a) {
+            const unsigned j = (unsigned)(kx[a] & 0xffffffffll);
+            u[a] = kx[a] != kInf ? row_of_entry(P, (long long)j) : 0;
+            v[a] = kx[a] != kInf ? __ldg(P.nlist + j) : 0;
+        }
+#pragma unroll
+        for (int a = 0; a < 4; ++a) {
+            if (kx[a] == kInf) continue;
+            const long long i = i0 + a * stride;
+            const long long x = set_of(R, i);
+            const int pu = find_root(D, u[a], false), pv = find_root(D, v[a], false);
+            const int q = (pu == (int)x) ? pv : pu;
+            const bool mutual = P.key[q] == kx[a];
+            P.tgt[i] = q | (mutual ? (int)0x80000000 : 0);
+        }
     }
 }
 
