@@ -67,11 +67,13 @@ __global__ void __launch_bounds__(256) k_dist_reps1(Params P, const int* R, long
                                                     const long long* buf) {
     const long long stride = (long long)gridDim.x * blockDim.x;
     const DS D = ds_of(P);
-    // four sets per thread in flight: each is a chain of dependent loads
-    // (row search, nlist, two finds, the other end's key)
+    // four sets per thread in flight: each is a chain of dependent loads.
+    // x holds one end of its edge j = (row(j), nlist[j]); when set(nlist[j])
+    // is not x the other end is that set and the row search (about four
+    // dependent loads) is skipped -- about half the sets
     for (long long i0 = lo + (long long)blockIdx.x * blockDim.x + threadIdx.x; i0 < hi; i0 += 4 * stride) {
         long long kx[4];
-        int u[4], v[4];
+        int pv[4];
 #pragma unroll
         for (int a = 0; a < 4; ++a) {
             const long long i = i0 + a * stride;
@@ -80,16 +82,15 @@ __global__ void __launch_bounds__(256) k_dist_reps1(Params P, const int* R, long
 #pragma unroll
         for (int a = 0; a < 4; ++a) {
             const unsigned j = (unsigned)(kx[a] & 0xffffffffll);
-            u[a] = kx[a] != kInf ? row_of_entry(P, (long long)j) : 0;
-            v[a] = kx[a] != kInf ? __ldg(P.nlist + j) : 0;
+            pv[a] = kx[a] != kInf ? find_root(D, __ldg(P.nlist + j), false) : 0;
         }
 #pragma unroll
         for (int a = 0; a < 4; ++a) {
             if (kx[a] == kInf) continue;
             const long long i = i0 + a * stride;
             const long long x = set_of(R, i);
-            const int pu = find_root(D, u[a], false), pv = find_root(D, v[a], false);
-            const int q = (pu == (int)x) ? pv : pu;
+            int q = pv[a];
+            if (q == (int)x) q = find_root(D, row_of_entry(P, kx[a] & 0xffffffffll), false);
             const bool mutual = P.key[q] == kx[a];
             P.tgt[i] = q | (mutual ? (int)0x80000000 : 0);
         }
@@ -497,26 +498,24 @@ __global__ void __launch_bounds__(kBlock, 2) k_dist_loop(Params P0, DistLoop DL)
         const DS D = ds_of(P0);
         for (long long i0 = gtid; i0 < nR; i0 += 4 * gstride) {
             long long kx[4];
-            unsigned j[4];
-            int u[4], v[4];
+            int pv[4];
 #pragma unroll
             for (int a = 0; a < 4; ++a) {
                 const long long i = i0 + a * gstride;
                 kx[a] = i < nR ? DL.buf[i] : kInf;
-                j[a] = (unsigned)(kx[a] & 0xffffffffll);
             }
 #pragma unroll
-            for (int a = 0; a < 4; ++a) {
-                u[a] = kx[a] != kInf ? row_of_entry(P0, (long long)j[a]) : 0;
-                v[a] = kx[a] != kInf ? __ldg(P0.nlist + j[a]) : 0;
+            for (int a = 0; a < 4; ++a) {   // (as k_dist_reps1: the row search only when set(v) == x)
+                const unsigned j = (unsigned)(kx[a] & 0xffffffffll);
+                pv[a] = kx[a] != kInf ? find_root(D, __ldg(P0.nlist + j), false) : 0;
             }
 #pragma unroll
             for (int a = 0; a < 4; ++a) {
                 if (kx[a] == kInf) continue;
                 const long long i = i0 + a * gstride;
                 const long long x = set_of(R, i);
-                const int pu = find_root(D, u[a], false), pv = find_root(D, v[a], false);
-                const int q = (pu == (int)x) ? pv : pu;
+                int q = pv[a];
+                if (q == (int)x) q = find_root(D, row_of_entry(P0, kx[a] & 0xffffffffll), false);
                 P0.tgt[i] = q | (__ldcg(P0.key + q) == kx[a] ? (int)0x80000000 : 0);
             }
         }
