@@ -654,6 +654,12 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
     // the populate output of this CTA: regions w = b, b + G, ... (region mode)
     const RegionSrcT<SOA> R = region_src<SOA>(P, b, s_pre, s_rcnt, s_red, &st->live[g], PH == 1);
     if (b0 && tid == 0 && PH == 2) st->phase2_round = g;
+    if (P.trace && tid == 0 && PH == 1) {   // diagnostics: this CTA's SM and its first pass's chunks
+        unsigned sm;
+        asm volatile("mov.u32 %0, %%smid;" : "=r"(sm));
+        P.trace[b] = sm;
+        P.trace[kMaxGrid + b] = R.nloc;
+    }
     trace_cta(P, 4 + 2 * g);
     grid.sync();
     __shared__ long long s_acc[kWarps][2];   // per warp: MSF weight, MSF edges (pass B)

@@ -67,6 +67,30 @@ def main():
               f"mean wait {wait:7.1f}")
         prev = end
     print(f"  sum of mean CTA wait at barriers: {tot_wait:.1f} us")
+    # what the slow CTAs of the first passes have in common: their SM, their work
+    G = st["grid"]
+    sm, nloc = tr[0][:G], tr[1][:G]
+    if float(sm.max()) > 0:
+        for slot in (5, 6, 7):
+            if not t[slot - 1] or not t[slot]:
+                continue
+            end = (tr[slot][:G] - t[slot - 1]) / 1e3
+            order = torch.argsort(end)
+            slow, fast = order[-G // 8:], order[: G // 8]
+            c = torch.corrcoef(torch.stack([end, nloc]))[0, 1]
+            print(f"  slot {slot}: end min {float(end.min()):.1f} med {float(end.median()):.1f} max {float(end.max()):.1f} us;"
+                  f" corr(end, first-pass chunks) {float(c):.2f}; slowest 1/8 chunks {float(nloc[slow].mean()):.0f}"
+                  f" vs fastest {float(nloc[fast].mean()):.0f}")
+            per_sm = {}
+            for b in range(G):
+                per_sm.setdefault(int(sm[b]), []).append(float(end[b]))
+            sms = sorted(per_sm)
+            means = torch.tensor([sum(per_sm[s]) / len(per_sm[s]) for s in sms])
+            print(f"    per-SM mean end: min {float(means.min()):.1f} max {float(means.max()):.1f}; slowest SMs "
+                  f"{[sms[i] for i in torch.argsort(means)[-8:].tolist()]}, fastest {[sms[i] for i in torch.argsort(means)[:8].tolist()]}")
+            half = len(sms) // 2
+            print(f"    SM ids < {sms[half]}: {float(means[:half].mean()):.1f} us, >=: {float(means[half:].mean()):.1f} us; "
+                  f"by SM id in 8 groups {[round(float(x), 0) for x in means[: len(means) // 8 * 8].view(8, -1).mean(1)]}")
 
 
 if __name__ == "__main__":
