@@ -26,13 +26,23 @@ constexpr int kStagePieces = 8;                // host path: CSR pieces uploaded
 constexpr int kSplitSamples = 512;             // crowded-round threshold: about this many samples
 constexpr int kSplitSampleSlots = 1024;        // sample slots (max(1, 512 / G) per CTA, first CTAs)
 constexpr int kQBins = 2048;                   // exact-quantile radix select: 11 + 11 + 10 bits
+#ifndef ECL_POP_DYN
+#define ECL_POP_DYN 2                          // populate: dynamic tail in phase 2 (bit 1; phase 1 keeps its
+                                               // contiguous slices: C5 populate1 8.45 -> 9.83 ms with it)
+#endif
+#ifndef ECL_POP_BATCH
+#define ECL_POP_BATCH 8                        // chunks per dynamic claim
+#endif
+#ifndef ECL_POP_STATIC
+#define ECL_POP_STATIC 4                       // static share of each warp's chunks, in eighths
+#endif
 constexpr int kMaxLevels = 24;                 // relabel: contraction levels (level 0 = the vertices)
 static_assert(kMaxGrid == ECL_MST_TRACE_CTAS, "trace layout");
 
 struct Internal {
     unsigned long long reps;           // distributed path: sets with a finite key this round
     long long nroots;                  // distributed path: size of the next round's root list
-    unsigned int done;                 // unused ticket
+    unsigned int pop_ctr[2];           // populate<PH>: dynamic batches claimed (ECL_POP_DYN)
     int g_cur;                         // first global round of the running phase
     int g_end;                         // last global round of the finished phase
     int giant;                         // root of the largest set after phase 1 (-1: none)
@@ -69,7 +79,7 @@ static inline long long ceil_div(long long a, long long b) { return (a + b - 1) 
 static inline long long wl_capacity(long long M) {
     const long long nchunks = ceil_div(M, kChunk);
     const long long wmax = nchunks < kMaxPopWarps ? nchunks : kMaxPopWarps;
-    return (nchunks + wmax) * (long long)kChunk;
+    return (nchunks + 3 * wmax) * (long long)kChunk;   // (2 wmax: slack of the populate's dynamic tail)
 }
 
 // dup: worklist copies per canonical edge (2 for opts.both_directions)
@@ -107,6 +117,9 @@ struct Params {
     long long rcap;                   // tuples per region
     int pop_contig;                   // bit PH-1: populate<PH> walks contiguous slices of rcap/kChunk chunks
     int pop_cta0;                     // first populate CTA of this launch (staged host path: pieces)
+    long long pop_span;               // chunks per warp of the contiguous order without a dynamic tail
+    int pop_dyn;                      // bit PH-1: populate<PH> ends with dynamically claimed batches
+    int pop_s0;                       // ... after this many static chunks per warp
     const long long* __restrict__ nindex;
     const int* __restrict__ nlist;
     const int* __restrict__ eweight;

@@ -299,8 +299,23 @@ static int run_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t
         case 3: contig = 1; break;
         default: contig = 1; break;
     }
+    // dynamic tail (ECL_POP_DYN, bit PH-1): each populate warp walks a static
+    // share of ECL_POP_STATIC/8 of its chunks, then claims batches of
+    // ECL_POP_BATCH chunks from one counter until none are left.  The warps
+    // of an SM do not progress at one rate (the scheduler favours the oldest
+    // CTAs: on C5 the populate-2 CTAs of the four residency slots ended at
+    // 8.6, 9.2, 10.3 and 11.8 ms), so a fixed split leaves the GPU draining.
+    // A warp claims only while its region keeps room for everything it may
+    // still hold; regions get 2 B + 4 chunks of slack, which guarantees that
+    // the claims never stall with chunks left.  Off for the
+    // staged host path's phase 1 (a piece may not have landed yet) and the
+    // thread-based populate.
+    const long long span = ceil_div(nchunks, W);
+    const long long dup = o.both_directions ? 2 : 1;
+    int dyn = (o.populate_mode == 1 ? 0 : ECL_POP_DYN) & (stg ? 2 : 3);
+    if (dyn && (span + 2 * ECL_POP_BATCH + 4) * W * kChunk * dup > L.wl_cap) dyn = 0;   // no room for the slack
     // (both_directions: every candidate edge takes two tuples)
-    const long long rcap = ceil_div(nchunks, W) * kChunk * (o.both_directions ? 2 : 1);
+    const long long rcap = (span + (dyn ? 2 * ECL_POP_BATCH + 4 : 0)) * kChunk * dup;
     // only warps that own a block write a region
     if (W * rcap > L.wl_cap) return fail(ECL_MST_ERR_WORKSPACE, "internal: regions exceed worklist capacity");
     // k_rounds arenas: the worklist of CTA b never exceeds its first input,
@@ -319,6 +334,9 @@ static int run_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t
     P.rcap = rcap;
     P.pop_contig = contig;
     P.pop_cta0 = 0;
+    P.pop_span = span;
+    P.pop_dyn = dyn;
+    P.pop_s0 = (int)(nchunks * ECL_POP_STATIC / 8 / W);
     P.nindex = reinterpret_cast<const long long*>(nindex);
     P.nlist = nlist;
     P.eweight = eweight;
@@ -428,7 +446,6 @@ static int run_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t
             e = cudaMemcpyAsync(const_cast<int32_t*>(eweight), stg->h_w, sizeof(int32_t) * (size_t)M,
                                 cudaMemcpyHostToDevice, stg->copy);
         if (e == cudaSuccess) e = cudaEventRecord(stg->ev[0], stg->copy);
-        const long long span = rcap / kChunk;
         for (int k = 0; k < pieces && e == cudaSuccess; ++k) {
             long long e0 = staged ? std::min<long long>(M, group_cta(k) * kPopWarps * span * kChunk) : 0;
             long long e1 = staged ? std::min<long long>(M, group_cta(k + 1) * kPopWarps * span * kChunk) : M;
@@ -947,6 +964,8 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
         P.cap = cap;
         P.W = (int)W;
         P.rcap = rcap;
+        P.pop_span = rcap / kChunk;
+        P.pop_dyn = 0;
         P.pop_contig = 1;   // phase 1: each warp a contiguous slice of the shard's chunks (as on one GPU)
         P.nindex = reinterpret_cast<const long long*>(nindex);
         P.nlist = nlist;

@@ -3,6 +3,8 @@
 // cycle filter).
 #pragma once
 
+#include <type_traits>
+
 #include "common.cuh"
 
 namespace eclmst {
@@ -73,7 +75,7 @@ __global__ void __launch_bounds__(256) k_init(Params P) {
             if (P.nindex[0] != 0 || P.nindex[P.n] != P.M) err = true;
             P.in->g_cur = 0;
             P.in->g_end = 0;
-            P.in->done = 0;
+            P.in->pop_ctr[0] = P.in->pop_ctr[1] = 0;
             P.in->giant = -1;
             P.in->splits = 0;
             P.in->tcount = P.in->tcanon = P.in->theavy = 0;
@@ -295,24 +297,83 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
         return x;
     };
     // the warp's chunks: interleaved w, w + W, ... or the contiguous slice
-    // [w B, (w + 1) B) with B = rcap / kChunk (see P.pop_contig)
+    // [w B, (w + 1) B) with B = P.pop_span (see P.pop_contig).  Phase 2 may
+    // end with a dynamic tail (P.pop_dyn): each warp walks only its first
+    // P.pop_s0 chunks, then claims batches of ECL_POP_BATCH chunks from
+    // P.in->pop_ctr (ecl_mst.cu says why).  (Phase 1 keeps the static order:
+    // its contiguous slices beat the balanced dynamic tail.)
+    constexpr bool DYNK = PH == 2;
     const bool contig = (P.pop_contig >> (PH - 1)) & 1;
-    const long long span = P.rcap / kChunk / (BOTH ? 2 : 1);   // chunks per warp (regions hold 2 copies)
+    const long long span = P.pop_span;
     const long long step = contig ? 1 : P.W;
-    const long long lc0 = contig ? (long long)w * span : w;
-    const long long lend = contig ? min(lc0 + span, P.nlocal) : P.nlocal;
+    const long long lend = contig ? min((long long)(w + 1) * span, P.nlocal) : P.nlocal;
     auto nxt = [&](long long lc) { return lc + step; };
-    if (lc0 < lend) {
+    // dynamic sequence (phase 2); chunk ids fit int32 (M < 2^32)
+    const bool dyn = DYNK && ((P.pop_dyn >> (PH - 1)) & 1);
+    const int nloc = (int)P.nlocal;
+    const int ws0 = dyn ? P.pop_s0 * P.W : 0;   // first dynamic chunk
+    int cur = 0, end = 0;   // the range being handed out (static: step W when interleaved)
+    if (DYNK) {
+        if (dyn) {
+            cur = contig ? w * P.pop_s0 : w;
+            end = contig ? cur + P.pop_s0 : ws0;
+        } else {
+            cur = contig ? (int)min((long long)w * span, P.nlocal) : w;
+            end = (int)lend;
+        }
+    }
+    // the next batch, claimed one batch ahead (lane 0's raw ticket; read only
+    // when needed, so the atomic's latency hides behind a batch of chunks)
+    unsigned tk_raw = 0;
+    bool tk = false;
+    const int tup = kChunk * (BOTH ? 2 : 1);   // tuples a chunk may add
+    auto claim = [&]() {
+        // room for the pipeline (up to 3 chunks), the rest of the current
+        // batch and the claimed one
+        tk = cnt + (2 * ECL_POP_BATCH + 3) * tup <= P.rcap;
+        if (tk && lane == 0) tk_raw = atomicAdd(&P.in->pop_ctr[PH - 1], (unsigned)ECL_POP_BATCH);
+    };
+    auto take = [&]() -> int {
+        if (cur < end) {
+            const int r = cur;
+            cur += (!contig && (!dyn || r < ws0)) ? P.W : 1;
+            return r;
+        }
+        if (!dyn) return -1;
+        if (!tk) claim();
+        if (!tk) return -1;
+        const int b = ws0 + (int)__shfl_sync(kFull, tk_raw, 0);
+        if (b >= nloc) {
+            tk = false;
+            cur = end = nloc;
+            return -1;
+        }
+        cur = b + 1;
+        end = min(b + ECL_POP_BATCH, nloc);
+        claim();
+        return b;
+    };
+    // (chunk indices: int in the dynamic phase, where registers are tight)
+    using cidx = typename std::conditional<DYNK, int, long long>::type;
+    const cidx lc0 = DYNK ? (cidx)take() : (cidx)(contig ? (long long)w * span : w);
+    cidx lq2 = -1;   // deep, dynamic: the chunk after the next one
+    if (DYNK ? lc0 >= 0 : lc0 < lend) {
         bracket(lc0, nr0, nrl);
         load_entries(P.shard + lc0 * P.nshards, nv, nw);
         if (deep) {
             starts(nr0, nrl, nsa, nsz);
             nrw = rowwords(nr0, nrl);
-            if (nxt(lc0) < lend) bracket(nxt(lc0), n2r0, n2rl);
+            if (DYNK) {
+                lq2 = take();
+                if (lq2 >= 0) bracket(lq2, n2r0, n2rl);
+            } else if (nxt(lc0) < lend) {
+                bracket(nxt(lc0), n2r0, n2rl);
+            }
         }
         nvb = vbits(nv, nw, nr0);
     }
-    for (long long lc = lc0; lc < lend; lc = nxt(lc)) {
+    cidx lc_next = -1;
+    for (cidx lc = lc0; DYNK ? lc >= 0 : lc < lend;) {
     const long long c = P.shard + lc * P.nshards;
     bool keep[kItems];
     int4 t[kItems];
@@ -333,19 +394,26 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
             vv[k] = nv[k];
             ww[k] = nw[k];
         }
-        const long long lcn = nxt(lc);
-        if (lcn < lend) {
+        const cidx lcn = DYNK ? (deep ? lq2 : (cidx)take()) : (cidx)nxt(lc);
+        const bool has_next = DYNK ? lcn >= 0 : lcn < lend;
+        if (has_next) {
             load_entries(P.shard + lcn * P.nshards, nv, nw);
             if (deep) {
                 nr0 = n2r0;
                 nrl = n2rl;
                 starts(nr0, nrl, nsa, nsz);
                 nrw = rowwords(nr0, nrl);
-                if (nxt(lcn) < lend) bracket(nxt(lcn), n2r0, n2rl);
+                if (DYNK) {
+                    lq2 = take();
+                    if (lq2 >= 0) bracket(lq2, n2r0, n2rl);
+                } else if (nxt(lcn) < lend) {
+                    bracket(nxt(lcn), n2r0, n2rl);
+                }
             } else {
                 bracket(lcn, nr0, nrl);
             }
         }
+        lc_next = has_next ? lcn : -1;
         int* mark = s_mark[warp];
 #pragma unroll
         for (int i = lane; i < kChunk; i += 32) mark[i] = -1;
@@ -396,7 +464,7 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
 #if ECL_EARLY_VBITS
         // the next chunk's far-end bits, issued half a chunk earlier than at
         // the end of this one (its entries have arrived by now)
-        if (PH == 2 && lcn < lend) nvb = vbits(nv, nw, nr0);
+        if (PH == 2 && has_next) nvb = vbits(nv, nw, nr0);
 #endif
         bool cand[kItems];
 #pragma unroll
@@ -489,7 +557,7 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
         }
     }
 #if !ECL_EARLY_VBITS
-    if (PH == 2 && nxt(lc) < lend) nvb = vbits(nv, nw, nr0);   // next chunk's far-end bits
+    if (PH == 2 && lc_next >= 0) nvb = vbits(nv, nw, nr0);   // next chunk's far-end bits
 #endif
     // L7: append the chunk's tuples to the warp's region (both_directions:
     // then their mirror copies <q, p, w, id>)
@@ -510,6 +578,7 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
             if (keep[i]) tst_cg<SOA>(out, cnt + off[i] + __popc(m[i] & lt), t[i], P.wlcap);
         cnt += tot;
     }
+    lc = DYNK ? lc_next : (cidx)nxt(lc);
     }
     if (err) atomicExch(&P.st->status, ECL_MST_ERR_INPUT);
     if (PH == 2 && kg >= 0) {
@@ -522,6 +591,13 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
         heavy_cnt = warp_sum(heavy_cnt);
     }
     if (lane == 0) P.region[w] = make_int4(cnt, canon_cnt, heavy_cnt, 0);
+    if (P.trace && lane == 0 && blockIdx.x < kMaxGrid / 2) {   // diagnostics: this CTA's last warp end, its SM
+        unsigned sm;
+        asm volatile("mov.u32 %0, %%smid;" : "=r"(sm));
+        atomicMax(reinterpret_cast<unsigned long long*>(P.trace + (PH == 1 ? 2 : 3) * kMaxGrid + blockIdx.x),
+                  globaltimer_ns());
+        P.trace[(long long)(PH == 1 ? 2 : 3) * kMaxGrid + kMaxGrid / 2 + blockIdx.x] = sm;
+    }
 }
 
 // ---------------------------------------------------------------------------

@@ -507,3 +507,25 @@ def test_contraction_levels(eclmst, seed):
         assert st["relabels"] >= 1, opts
     st = assert_parity(eclmst, G.path_graph(50_000), relabel=1)     # monotone path: one hook chain
     assert st["relabels"] >= 1
+
+
+@pytest.mark.parametrize("both", [0, 1])
+@pytest.mark.parametrize("seed", [0, 1])
+def test_populate_dynamic_tail_full_regions(eclmst, both, seed):
+    """The phase-2 populate's dynamic tail (ECL_POP_DYN) when every entry is
+    kept: a one-direction CSR (only u < v entries, reading Q11) whose edges
+    are all heavy (threshold below every weight), so phase 1 hooks nothing
+    and phase 2 emits a tuple per entry (two with both_directions).  Regions
+    fill up, and a warp that claims batches must stop at its room (rcap) --
+    every chunk still gets processed exactly once."""
+    gen = torch.Generator().manual_seed(4100 + seed)
+    n, m = 1 << 20, 4_300_000
+    u = torch.randint(0, n, (m,), generator=gen)
+    v = torch.randint(0, n, (m,), generator=gen)
+    lo, hi = torch.minimum(u, v), torch.maximum(u, v)
+    w = torch.randint(-(1 << 30), 1 << 30, (m,), generator=gen)
+    g = G.csr_from_entries(n, lo, hi, w, name=f"onedir{seed}")
+    stats = assert_parity(eclmst, g, filter=1, threshold_mode=1, threshold=-(1 << 31), both_directions=both)
+    assert stats["filtered"] == 1 and stats["phase2_round"] >= 0
+    # phase 2 kept every canonical entry but the self-loops
+    assert stats["live"][stats["phase2_round"]] == int((lo != hi).sum()) * (1 + both)

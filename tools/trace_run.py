@@ -32,7 +32,7 @@ def main():
     kw = {k: int(v) for k, v in (o.split("=") for o in args.opt)}
     kw["trace"] = 1
     opts = eclmst.default_options(**kw)
-    ws = torch.empty(eclmst.ecl_mst_workspace_bytes(g.n, g.M), dtype=torch.uint8, device=dev)
+    ws = torch.zeros(eclmst.ecl_mst_workspace_bytes(g.n, g.M), dtype=torch.uint8, device=dev)
     for _ in range(args.runs):
         eclmst.ecl_mst_device(g.n, g.nindex, g.nlist, g.eweight, workspace=ws, options=opts)
     st = eclmst.ecl_mst_read_stats(ws)
@@ -67,6 +67,28 @@ def main():
               f"mean wait {wait:7.1f}")
         prev = end
     print(f"  sum of mean CTA wait at barriers: {tot_wait:.1f} us")
+    # populate: per-CTA end (its last warp) and SM
+    trf = eclmst.ecl_mst_read_trace(ws, dict(st, grid=4096)).double()
+    KG = trf.shape[1]
+    for ph, slot, t0 in ((1, 2, t[1]), (2, 3, t[3])):
+        row, sms = trf[slot][: KG // 2], trf[slot][KG // 2:]
+        ok = row > t0 if t0 else row > 0
+        if not t0 or int(ok.sum()) == 0:
+            continue
+        end = (row[ok] - t0) / 1e3
+        sm_ok = sms[ok]
+        per = {}
+        for e, s_ in zip(end.tolist(), sm_ok.tolist()):
+            per.setdefault(int(s_), []).append(e)
+        sl = sorted(per)
+        mx = torch.tensor([max(per[s_]) for s_ in sl])
+        print(f"  populate{ph}: {int(ok.sum())} CTAs, end min {float(end.min()):.1f} med {float(end.median()):.1f} "
+              f"max {float(end.max()):.1f} us; per-SM last end min {float(mx.min()):.1f} max {float(mx.max()):.1f}; "
+              f"slowest SMs {[sl[i] for i in torch.argsort(mx)[-8:].tolist()]} fastest {[sl[i] for i in torch.argsort(mx)[:8].tolist()]}")
+        ne = end.numel() // 16 * 16
+        print(f"    by CTA index in 16 groups: {[round(float(x)) for x in end[:ne].view(16, -1).mean(1)]}")
+        print(f"    by CTA index mod 4: {[round(float(end[i::4].mean())) for i in range(4)]}; deciles "
+              f"{[round(float(x)) for x in torch.quantile(end, torch.linspace(0, 1, 11, dtype=end.dtype))]}")
     # what the slow CTAs of the first passes have in common: their SM, their work
     G = st["grid"]
     sm, nloc = tr[0][:G], tr[1][:G]
