@@ -193,10 +193,17 @@ static inline bool giant_bitmap_on(int32_t opt, int32_t n) {
 // (deep: phase 1 also prefetches the next chunk's row starts; measured on
 // C5, M = 2e9: populate1 8.73 -> 8.31 ms, but C4 +0.26 ms, C3 +0.05: only
 // from M >= 2^30 on)
+// (pack: the phase-2 populate works on its surviving candidates packed one
+// per lane -- it pays where few survive per chunk: graphs filtered by the
+// largest-set bitmap (C5 populate2 10.43 -> 10.05 ms) or whose heavy entries
+// are at most half of all (C3 0.545 -> 0.454 ms); on a dense graph without
+// the bitmap about half of every chunk survives, and the per-item path, whose
+// four setid loads per lane overlap, is faster (C4 2.33 vs 2.46 ms))
 template <int PH>
-static void (*pop_kernel(bool soa, int both, bool deep = false))(Params) {
+static void (*pop_kernel(bool soa, int both, bool deep = false, bool pack = false))(Params) {
     if (soa) return both ? k_populate<PH, true, true> : k_populate<PH, true, false>;
     if (both) return k_populate<PH, false, true>;
+    if (PH == 2 && pack && ECL_PACK2) return k_populate<PH, false, false, -1, true>;
     return (PH == 1 && deep) ? k_populate<PH, false, false, 1> : k_populate<PH, false, false>;
 }
 template <int PH>
@@ -515,7 +522,8 @@ static int run_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t
             else k_populate_thread<2, false><<<flat_blocks, 256, 0, s>>>(P);
             k_regions<2><<<1, 256, 0, s>>>(P);
         } else {
-            pop_kernel<2>(soa, P.both)<<<(unsigned)pop_blocks, kPopBlock, 0, s>>>(P);
+            const bool pack2 = P.giant_bits != nullptr || M <= 2LL * P.filter_c * n;
+            pop_kernel<2>(soa, P.both, false, pack2)<<<(unsigned)pop_blocks, kPopBlock, 0, s>>>(P);
         }
         e = cudaGetLastError();
     }

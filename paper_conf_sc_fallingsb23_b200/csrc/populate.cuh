@@ -177,7 +177,7 @@ __global__ void __launch_bounds__(1024) k_qselect(Params P) {
 // ---------------------------------------------------------------------------
 // k_populate<PH>: one warp per 128-entry CSR chunk
 // ---------------------------------------------------------------------------
-template <int PH, bool SOA = false, bool BOTH = false, int DEEP = -1>
+template <int PH, bool SOA = false, bool BOTH = false, int DEEP = -1, bool PK2 = false>
 #ifndef ECL_DEEP_PH1
 #define ECL_DEEP_PH1 0
 #endif
@@ -194,11 +194,19 @@ template <int PH, bool SOA = false, bool BOTH = false, int DEEP = -1>
 #define ECL_P2_GUARD_COLD 0   // phase-2 populate: guard the atomicMin of slots other than the giant's
                               // (off: C4 populate2 2.60 -> 2.40 ms, C5 11.8 -> 11.4 ms)
 #endif
+#ifndef ECL_PACK1
+#define ECL_PACK1 1   // phase 1: per-candidate work on packed candidates (C4 populate1 1.81 -> 1.48 ms)
+#endif
+#ifndef ECL_PACK2
+#define ECL_PACK2 1   // phase 2 packs when few candidates survive per chunk (see pop_kernel)
+#endif
 #ifndef ECL_POP_MINB
 #define ECL_POP_MINB 4
 #endif
 __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) {
     __shared__ int s_mark[kPopWarps][kChunk];
+    // packed candidates (PACK)
+    __shared__ int4 s_stage[(PH == 1 ? ECL_PACK1 : PK2) ? kPopWarps : 1][(PH == 1 ? ECL_PACK1 : PK2) ? kChunk : 1];
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     if (!input_ok(P)) return;   // k_init rejected nindex: rowstart[] is not valid
     if (PH == 2 && !phase2_needed(P)) return;
@@ -219,7 +227,9 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
     const int w = (P.pop_cta0 + (int)blockIdx.x) * kPopWarps + warp;
     if (w >= P.W) return;   // (sharded path: partial last CTA)
     int4* const out = tadd<SOA>(P.wl0, (long long)w * P.rcap);
-    int cnt = 0, canon_cnt = 0, heavy_cnt = 0;
+    int cnt = 0, canon_cnt = 0, heavy_cnt = 0, cand_tot = 0;
+    // PACK: per-candidate work on candidates packed one per lane (phase 1)
+    constexpr bool PACK = PH == 1 ? ECL_PACK1 != 0 : PK2;
     bool err = false;
     const int p0 = lane * kItems;
     // CSR entries of chunk c (lane owns entries p0 .. p0+3), streaming loads
@@ -476,12 +486,90 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
             const bool heavy = filtered && ww[k] >= T;                // L6 threshold condition
             if (PH == 1) {
                 canon_cnt += canon;
-                heavy_cnt += (canon && heavy);
+                if (!PACK) heavy_cnt += (canon && heavy);   // (packed: |canonical| - |candidates|)
                 cand[k] = canon && !heavy;
             } else {
                 cand[k] = canon && heavy;
             }
         }
+        int idx[kItems];   // packed position of each candidate (-1: none)
+        int tot = 0;
+        if constexpr (PACK) {
+            // The chunk's candidates, packed one per lane through shared
+            // memory: the per-candidate work below runs once per 32 of them
+            // instead of once per lane item (C5: about 6 candidates per 128
+            // entries in phase 1, and in phase 2 after the bitmap test).
+            if (PH == 2 && giant >= 0) {   // both ends in the largest set: filtered here
+#pragma unroll
+                for (int k = 0; k < kItems; ++k) {
+                    const int wi = (row[k] >> 5) - (r0 >> 5);
+                    const unsigned wd = __shfl_sync(kFull, rw, wi & 31);
+                    // (a row beyond the lanes' 32 words -- a chunk spanning
+                    // over 1024 rows -- counts as outside: its edge then takes
+                    // the setid path, which decides the same)
+                    const bool rin = deep && wi < 32 && ((wd >> (row[k] & 31)) & 1u);
+                    if (rin && ((vb >> k) & 1u)) cand[k] = false;
+                }
+            }
+            const unsigned lt = (1u << lane) - 1u;
+#pragma unroll
+            for (int k = 0; k < kItems; ++k) {
+                const unsigned m = __ballot_sync(kFull, cand[k]);
+                idx[k] = cand[k] ? tot + __popc(m & lt) : -1;
+                tot += __popc(m);
+            }
+            if (PH == 1) cand_tot += tot;
+        }
+        if constexpr (PACK) {
+            const unsigned lt = (1u << lane) - 1u;
+            int4* const stage = s_stage[warp];
+#pragma unroll
+            for (int k = 0; k < kItems; ++k)
+                if (idx[k] >= 0) stage[idx[k]] = make_int4(row[k], vv[k], ww[k], p0 + k);
+            __syncwarp();
+            for (int base = 0; base < tot; base += 32) {
+                const bool on = lane < tot - base;
+                int4 e = make_int4(0, 0, 0, 0);
+                bool kp = false;
+                if (on) {
+                    e = stage[base + lane];
+                    kp = true;
+                    if (PH == 2) {   // set(u), set(v): one load each after k_flatten
+                        e.x = __ldca(sid + e.x);
+                        e.y = __ldca(sid + e.y);
+                        if (!P.flatten) {
+                            e.x = find_root(D, e.x, P.halving != 0);
+                            e.y = find_root(D, e.y, P.halving != 0);
+                        }
+                        kp = e.x != e.y;                                 // phase 2: the filter
+                    }
+                }
+                const unsigned j = (unsigned)(c0 + e.w);
+                const long long key = make_key(e.z, j);                  // L19 val <- e_w : e_id
+                if (kp) {
+                    rec(e.x, key);                                       // L20-21
+                    rec(e.y, key);
+                    if (BOTH) {   // opts.both_directions: the mirror copy records it again
+                        rec(e.y, key);
+                        rec(e.x, key);
+                    }
+                }
+                // L7: append (phase 2: the kept ones, compacted)
+                const unsigned km = PH == 2 ? __ballot_sync(kFull, kp) : 0u;
+                const int at = PH == 2 ? __popc(km & lt) : lane;
+                const int4 tt = make_int4(e.x, e.y, e.z, (int)j);
+                if (kp) {
+                    if (BOTH) {
+                        tst_cg<SOA>(out, cnt + 2LL * at, tt, P.wlcap);
+                        tst_cg<SOA>(out, cnt + 2LL * at + 1, make_int4(e.y, e.x, e.z, (int)j), P.wlcap);
+                    } else {
+                        tst_cg<SOA>(out, cnt + at, tt, P.wlcap);
+                    }
+                }
+                cnt += (PH == 2 ? __popc(km) : min(32, tot - base)) * (BOTH ? 2 : 1);
+            }
+            __syncwarp();   // (the next chunk's stage)
+        } else {
         int pk[kItems], qk[kItems];
 #pragma unroll
         for (int k = 0; k < kItems; ++k) {
@@ -555,12 +643,14 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
                 }
             }
         }
+        }   // !PACK
     }
 #if !ECL_EARLY_VBITS
     if (PH == 2 && lc_next >= 0) nvb = vbits(nv, nw, nr0);   // next chunk's far-end bits
 #endif
     // L7: append the chunk's tuples to the warp's region (both_directions:
     // then their mirror copies <q, p, w, id>)
+    if constexpr (!PACK)
     for (int copy = 0; copy < 1 + BOTH; ++copy) {
         unsigned m[kItems];
         int off[kItems];
@@ -588,7 +678,7 @@ __global__ void __launch_bounds__(kPopBlock, ECL_POP_MINB) k_populate(Params P) 
     }
     if (PH == 1) {   // |E| and the deferred count of this warp's chunks
         canon_cnt = warp_sum(canon_cnt);
-        heavy_cnt = warp_sum(heavy_cnt);
+        heavy_cnt = PACK ? canon_cnt - cand_tot : warp_sum(heavy_cnt);
     }
     if (lane == 0) P.region[w] = make_int4(cnt, canon_cnt, heavy_cnt, 0);
     if (P.trace && lane == 0 && blockIdx.x < kMaxGrid / 2) {   // diagnostics: this CTA's last warp end, its SM

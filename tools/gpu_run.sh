@@ -13,7 +13,7 @@ for STEP in "$@"; do
   case $STEP in
     info) (nproc; free -g; nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv) > gpurun_out/${TAG}_info.txt 2>&1
           cat gpurun_out/${TAG}_info.txt;;
-    tests) timeout 2400 python -m pytest tests -q -x -m "gpu and not slow" > gpurun_out/${TAG}_pytest.txt 2>&1
+    tests) timeout 900 python -m pytest tests -q -x -m "gpu and not slow" > gpurun_out/${TAG}_pytest.txt 2>&1
            echo "tests rc=$?"; tail -3 gpurun_out/${TAG}_pytest.txt;;
     slow) timeout 3000 python -m pytest tests -q -x -m "gpu and slow" --durations=10 > gpurun_out/${TAG}_pytest_slow.txt 2>&1
           echo "slow rc=$?"; tail -15 gpurun_out/${TAG}_pytest_slow.txt;;
