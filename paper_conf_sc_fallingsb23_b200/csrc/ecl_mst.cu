@@ -199,12 +199,23 @@ static inline bool giant_bitmap_on(int32_t opt, int32_t n) {
 // are at most half of all (C3 0.545 -> 0.454 ms); on a dense graph without
 // the bitmap about half of every chunk survives, and the per-item path, whose
 // four setid loads per lane overlap, is faster (C4 2.33 vs 2.46 ms))
+// (deep: the next chunk's row starts and row-bitmap words are prefetched
+// too.  Phase 2 needs it for the largest-set bitmap, whose row bits come from
+// the prefetched words (C5 populate2 10.0 vs 15.9 ms without); elsewhere the
+// extra loads and registers cost more than they hide (C4 populate2 2.32 ->
+// 2.03 ms without; phase 1 of C5 8.11 -> 7.72 ms without, with packing))
+#ifndef ECL_DEEP_PH1_M
+#define ECL_DEEP_PH1_M (1LL << 62)   // phase 1 deep from this M on (never)
+#endif
 template <int PH>
 static void (*pop_kernel(bool soa, int both, bool deep = false, bool pack = false))(Params) {
     if (soa) return both ? k_populate<PH, true, true> : k_populate<PH, true, false>;
     if (both) return k_populate<PH, false, true>;
-    if (PH == 2 && pack && ECL_PACK2) return k_populate<PH, false, false, -1, true>;
-    return (PH == 1 && deep) ? k_populate<PH, false, false, 1> : k_populate<PH, false, false>;
+    if (PH == 2) {
+        if (pack && ECL_PACK2) return deep ? k_populate<PH, false, false, 1, true> : k_populate<PH, false, false, 0, true>;
+        return deep ? k_populate<PH, false, false, 1> : k_populate<PH, false, false, 0>;
+    }
+    return deep ? k_populate<PH, false, false, 1> : k_populate<PH, false, false, 0>;
 }
 template <int PH>
 static const void* rounds_kernel(bool soa, int drive) {
@@ -497,7 +508,7 @@ static int run_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t
             k_regions<1><<<1, 256, 0, s>>>(P);
             e = cudaGetLastError();
         } else {
-            pop_kernel<1>(soa, P.both, M >= (1LL << 30))<<<(unsigned)pop_blocks, kPopBlock, 0, s>>>(P);
+            pop_kernel<1>(soa, P.both, M >= ECL_DEEP_PH1_M)<<<(unsigned)pop_blocks, kPopBlock, 0, s>>>(P);
             e = cudaGetLastError();
         }
     }
@@ -523,7 +534,7 @@ static int run_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t
             k_regions<2><<<1, 256, 0, s>>>(P);
         } else {
             const bool pack2 = P.giant_bits != nullptr || M <= 2LL * P.filter_c * n;
-            pop_kernel<2>(soa, P.both, false, pack2)<<<(unsigned)pop_blocks, kPopBlock, 0, s>>>(P);
+            pop_kernel<2>(soa, P.both, P.giant_bits != nullptr, pack2)<<<(unsigned)pop_blocks, kPopBlock, 0, s>>>(P);
         }
         e = cudaGetLastError();
     }
