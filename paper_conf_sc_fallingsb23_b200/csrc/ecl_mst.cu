@@ -217,6 +217,11 @@ static void (*pop_kernel(bool soa, int both, bool deep = false, bool pack = fals
     }
     return deep ? k_populate<PH, false, false, 1> : k_populate<PH, false, false, 0>;
 }
+// the phase-2 populate a parameter set takes (single-GPU rule, see run_device)
+static void (*pop2(const Params& P))(Params) {
+    const bool pack2 = P.giant_bits != nullptr || P.M <= 2LL * P.filter_c * P.n;
+    return pop_kernel<2>(false, 0, P.giant_bits != nullptr, pack2);
+}
 template <int PH>
 static const void* rounds_kernel(bool soa, int drive) {
     if (soa) {
@@ -1128,7 +1133,7 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
             if (e == cudaSuccess) e = cudaStreamSynchronize(s);
             if (e != cudaSuccess) return fail(ECL_MST_ERR_CUDA, "phase2: %s", cudaGetErrorString(e));
             const long long nroots = reinterpret_cast<volatile long long*>(h->h_map)[1];
-            for (int k = 0; k < S; ++k) k_populate<2><<<(unsigned)ceil_div(sp[k].W, kPopWarps), kPopBlock, 0, s>>>(sp[k]);
+            for (int k = 0; k < S; ++k) pop2(sp[k])<<<(unsigned)ceil_div(sp[k].W, kPopWarps), kPopBlock, 0, s>>>(sp[k]);
             if ((rc = check("populate2"))) return rc;
             if ((rc = run_loop(2, g, rlist[0], nroots, rlist[1], rlist[0]))) return rc;
         }
@@ -1157,7 +1162,7 @@ int ecl_mst_dist_device(void* handle, int32_t local_shards, int32_t n, int64_t M
         }
         for (int k = 0; k < S; ++k) {
             if (ph == 1) k_populate<1><<<(unsigned)ceil_div(sp[k].W, kPopWarps), kPopBlock, 0, s>>>(sp[k]);
-            else k_populate<2><<<(unsigned)ceil_div(sp[k].W, kPopWarps), kPopBlock, 0, s>>>(sp[k]);
+            else pop2(sp[k])<<<(unsigned)ceil_div(sp[k].W, kPopWarps), kPopBlock, 0, s>>>(sp[k]);
         }
         if ((rc = check("populate"))) return rc;
         bool first = true;
