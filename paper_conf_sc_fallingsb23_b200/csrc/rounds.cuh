@@ -442,6 +442,15 @@ __device__ __forceinline__ bool use_guard(const Params& P, long long live, long 
 #ifndef ECL_CROWD_RATIO
 #define ECL_CROWD_RATIO 6    // auto: split when live > this x last round's MSF edges (C5: 56.8 -> 54.6 ms vs 16)
 #endif
+#ifndef ECL_DRAIN_FLAT
+#define ECL_DRAIN_FLAT 1
+#endif
+#ifndef ECL_PREFLAT
+#define ECL_PREFLAT 1    // flatten a small open level before pass A when live >= this x its ids (0: never)
+#endif
+#ifndef ECL_DRAIN_FLAT_MAX
+#define ECL_DRAIN_FLAT_MAX (1LL << 22)   // open levels up to this many ids
+#endif
 #ifndef ECL_SPLIT_C
 #define ECL_SPLIT_C 2        // light part: about this many edges per MSF edge of the last round
                              // (4 -> 2: C4 7.18 -> 7.10 ms, C2 2.283 -> 2.262 ms, C5 -0.5%, C3 +-0)
@@ -758,6 +767,19 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
             }
         }
         __syncthreads();
+#if ECL_PREFLAT
+        // a small open level found by many more tuples than it has ids, after
+        // a round that hooked (chains of hooks make long finds): compress it
+        // first, every id in parallel, so that pass A's finds take one hop
+        if (!mapped && win > 0 && s_lv[1] <= ECL_DRAIN_FLAT_MAX && L >= ECL_PREFLAT * s_lv[1]) {
+            const long long lo = s_lv[0], hi = s_lv[0] + s_lv[1];
+            for (long long x = lo + (long long)blockIdx.x * kBlock + tid; x < hi; x += (long long)gridDim.x * kBlock) {
+                const int r = find_root(D, (int)x, true);
+                if (r != (int)x) __stcg(D.par(x), r);
+            }
+            grid.sync();
+        }
+#endif
         const bool guard = use_guard(P, L, win, s_lv[1]);
         // a split defers to the back of the output arena; with tuples already
         // deferred (hb >= 0) only when that is the same buffer, below them --
@@ -816,6 +838,20 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
         ++g;
         if (tid == 0) s_out = 0;
         __syncthreads();
+#if ECL_DRAIN_FLAT
+        // the deferred tuples' ends have not been found since the split, while
+        // the light part's rounds hooked chains of sets above them: compress
+        // the open level first (every id to its root, all ids in parallel),
+        // so that the drain's finds take one hop
+        if (s_lv[1] <= ECL_DRAIN_FLAT_MAX) {
+            const long long lo = s_lv[0], hi = s_lv[0] + s_lv[1];
+            for (long long x = lo + (long long)blockIdx.x * kBlock + tid; x < hi; x += (long long)gridDim.x * kBlock) {
+                const int r = find_root(D, (int)x, true);
+                if (r != (int)x) __stcg(D.par(x), r);
+            }
+            grid.sync();
+        }
+#endif
         passA(P, D, H, wl[ob], &s_out, true);
         cur = ob;
         __syncthreads();
