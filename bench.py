@@ -161,23 +161,25 @@ class ClockSampler:
 def algorithmic_bytes(n: int, M: int, st: dict) -> dict:
     """Bytes the method must move per launch, by kernel stage.
 
-    init        20 B/vertex  (nindex 8 read; parent 4 + best-edge key 8 written)
-    populate    8 B/CSR entry (nlist+eweight) + 8 B/vertex (nindex) [+1 B/entry in_mst, phase 1]
+    init        20 B/vertex  (nindex 8 read; parent 4 + best-edge key 8 written) + M/8 (MSF bit marks zeroed)
+    populate    8 B/CSR entry (nlist+eweight) + 8 B/vertex (nindex)
                 + per emitted tuple 16 B write + 2x8 B key atomicMin
                 [phase 2: + 2x4 B parent gathers per heavy canonical edge]
     flatten     8 B/vertex (parent read + write)
     rounds      pass A: per input tuple 16 B read + 2x4 B parent; per survivor 16 B write + 2x8 B key min
                 pass B: per tuple 16 B read + 2x8 B key reads; per winner 4 B hook + 8 B key reset + 1 B mark
+    finalize    1 B/CSR entry (in_mst, written once from the bit marks) + M/8 (the marks read)
     """
     live = st["live"]
     win = st["winners"]
     R = len(live)
     p2 = st["phase2_round"]
-    b = {"init": 20 * n, "populate1": 0, "rounds1": 0, "flatten": 0, "populate2": 0, "rounds2": 0}
+    b = {"init": 20 * n + M // 8, "populate1": 0, "rounds1": 0, "flatten": 0, "populate2": 0, "rounds2": 0,
+         "finalize": M + M // 8}
     for g in range(R):
         ph = "2" if (p2 >= 0 and g >= p2) else "1"
         if g == 0:
-            b["populate1"] += 8 * M + 8 * n + M + 32 * live[0]
+            b["populate1"] += 8 * M + 8 * n + 32 * live[0]
         elif g == p2:
             b["flatten"] += 8 * n
             b["populate2"] += 8 * M + 8 * n + 8 * st["heavy_edges"] + 32 * live[g]

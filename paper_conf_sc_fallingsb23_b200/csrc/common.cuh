@@ -66,7 +66,7 @@ struct Internal {
 };
 
 struct Layout {
-    size_t stats, internal, trace, rowstart, region, giant, samp, qhist, lvcnt, key, parent, setid, wl0, wl1, total;
+    size_t stats, internal, trace, rowstart, region, giant, samp, qhist, lvcnt, mbits, key, parent, setid, wl0, wl1, total;
     long long wl_cap;                  // tuples per worklist buffer
 };
 
@@ -97,6 +97,7 @@ static inline Layout layout_for(int64_t n, int64_t M, int dup = 1) {
     L.samp = off;     off = align_up(off + sizeof(int) * (size_t)kSplitSampleSlots, 256);
     L.qhist = off;    off = align_up(off + sizeof(unsigned long long) * (size_t)kQBins, 256);
     L.lvcnt = off;    off = align_up(off + sizeof(int) * (size_t)kMaxGrid, 256);
+    L.mbits = off;    off = align_up(off + sizeof(unsigned) * (size_t)((M + 31) / 32 + 1), 256);
     // key / parent: 2n slots, the vertices plus the contraction levels (Internal)
     L.key = off;      off = align_up(off + sizeof(long long) * (size_t)(2 * n), 256);
     L.parent = off;   off = align_up(off + sizeof(int) * (size_t)(2 * n), 256);
@@ -159,6 +160,7 @@ struct Params {
     int nshards;                      // total shards
     long long nlocal;                 // chunks of this shard: shard, shard + nshards, ...
     int zero_mst;                     // populate phase 1 zeroes its chunks of in_mst
+    unsigned* mbits;                  // MSF marks as bits (k_expand writes in_mst at the end), or null: bytes
     int* acnt;                        // per arena tuple count (distributed pass A)
     int* tgt;                         // per vertex hook target (distributed rep pass)
     long long* const* keys_all;       // virtual shards: every shard's key array
@@ -211,6 +213,15 @@ __device__ __forceinline__ bool input_ok(const Params& P) {
 // phase 2 runs iff filtering is on and phase 1 deferred at least one edge
 // (read-only within the kernels that ask: one L1 line per SM, not one L2
 // slice hammered by every warp of the grid)
+// L31: edge id joins the MSF.  With P.mbits a bit (a fire-and-forget RED.OR
+// into M/8 bytes, which the L2 holds far better than a random byte store
+// into the M-byte in_mst, a DRAM read-modify-write of a sector on C5);
+// k_expand writes in_mst from the bits at the end.
+__device__ __forceinline__ void mark_msf(const Params& P, unsigned id) {
+    if (P.mbits) atomicOr(P.mbits + (id >> 5), 1u << (id & 31));
+    else P.in_mst[id] = 1;
+}
+
 __device__ __forceinline__ bool phase2_needed(const Params& P) {
     return __ldg(&P.st->filtered) != 0 && __ldg(&P.st->heavy_edges) != 0 && __ldg(&P.st->status) == 0;
 }

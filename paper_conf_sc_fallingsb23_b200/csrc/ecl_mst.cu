@@ -184,6 +184,9 @@ static inline int round_bound_for(int32_t n) {
 }
 
 // opts.giant_bitmap: -1 auto (parent[] beyond about half the L2), 0 off, 1 on
+#ifndef ECL_MSF_BITS
+#define ECL_MSF_BITS 1
+#endif
 static inline bool giant_bitmap_on(int32_t opt, int32_t n) {
     return opt > 0 || (opt < 0 && (long long)n >= ECL_GIANT_MIN_N);
 }
@@ -406,7 +409,9 @@ static int run_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t
     P.shard = 0;
     P.nshards = 1;
     P.nlocal = nchunks;
-    P.zero_mst = 1;
+    // MSF marks as bits, in_mst written once at the end (ECL_MSF_BITS; see mark_msf)
+    P.mbits = ECL_MSF_BITS ? reinterpret_cast<unsigned*>(ws + L.mbits) : nullptr;
+    P.zero_mst = P.mbits ? 0 : 1;
     P.acnt = nullptr;
     P.tgt = nullptr;
     P.hcnt = nullptr;
@@ -548,6 +553,7 @@ static int run_device(int32_t n, int64_t M, const int64_t* nindex, const int32_t
         e = cudaLaunchCooperativeKernel(rounds_kernel<2>(soa, P.drive), dim3((unsigned)G), dim3(kBlock), args, 0, s);
     if (e == cudaSuccess) e = mark();
     if (e == cudaSuccess) {
+        if (P.mbits) k_expand<<<(unsigned)std::max<long long>(1, std::min<long long>(ceil_div(M / 16, 256), (long long)di.sms * 8)), 256, 0, s>>>(P);
         k_finalize<<<1, 32, 0, s>>>(P);
         e = cudaGetLastError();
     }

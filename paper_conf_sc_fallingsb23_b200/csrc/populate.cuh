@@ -36,6 +36,8 @@ __global__ void __launch_bounds__(256) k_init(Params P) {
         }
         for (long long c = (s + kChunk - 1) / kChunk; c * kChunk < e && c < P.nchunks; ++c) P.rowstart[c] = (int)v;
     }
+    if (P.mbits)   // no edge in the MSF yet (the bit marks of mark_msf)
+        for (long long i = i0; i < (P.M + 31) / 32; i += stride) P.mbits[i] = 0u;
     if (blockIdx.x == 0) {
         ecl_mst_stats* st = P.st;   // zeroed by a memset node just before this kernel
         __shared__ int s_w[kMaxSamples];

@@ -390,7 +390,7 @@ __device__ __forceinline__ void passB(const Params& P, const DS& D, const SRC& S
                 if (wq && !(wp && q < p)) __stcg(D.par(q), p);
                 if (!NORESET && wp) __stcg(D.k(p), kInf);              // L35
                 if (!NORESET && wq) __stcg(D.k(q), kInf);              // L36
-                P.in_mst[(unsigned)t[i].w] = 1;                        // L31
+                mark_msf(P, (unsigned)t[i].w);                         // L31
                 // (both_directions: the edge's two copies make the same
                 // hooks and marks; only the p < q copy counts it)
                 if (!P.both || p < q) {
@@ -894,6 +894,38 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
         st->rounds = g + 1;
         st->refilters = __ldcg(&P.in->splits);
         if (overflow) atomicExch(&st->status, ECL_MST_ERR_ROUNDS);
+    }
+}
+
+// in_mst from the bit marks (P.mbits): 16 bytes per thread (4 where in_mst is
+// not 16-byte aligned), coalesced.  Every byte of in_mst is written here, once
+// (Alg. 1's "not in MST" included).
+__device__ __forceinline__ unsigned expand4(unsigned b) {   // 4 bits -> 4 bytes 0/1
+    return (b & 1u) | ((b & 2u) << 7) | ((b & 4u) << 14) | ((b & 8u) << 21);
+}
+__global__ void __launch_bounds__(256) k_expand(Params P) {
+    const long long stride = (long long)gridDim.x * blockDim.x;
+    const long long t0 = (long long)blockIdx.x * blockDim.x + threadIdx.x;
+    long long done = 0;   // bytes written by the vector loop
+    if ((reinterpret_cast<uintptr_t>(P.in_mst) & 15) == 0) {
+        const long long n16 = P.M / 16;
+        for (long long i = t0; i < n16; i += stride) {
+            const unsigned b = (__ldg(P.mbits + (i >> 1)) >> ((i & 1) * 16)) & 0xFFFFu;
+            __stcs(reinterpret_cast<uint4*>(P.in_mst) + i,
+                   make_uint4(expand4(b), expand4(b >> 4), expand4(b >> 8), expand4(b >> 12)));
+        }
+        done = n16 * 16;
+    } else {
+        const long long n4 = P.M / 4;
+        for (long long i = t0; i < n4; i += stride) {
+            const unsigned b = (__ldg(P.mbits + (i >> 3)) >> ((i & 7) * 4)) & 0xFu;
+            __stcs(reinterpret_cast<unsigned*>(P.in_mst) + i, expand4(b));
+        }
+        done = n4 * 4;
+    }
+    if (blockIdx.x == 0 && threadIdx.x < P.M - done) {
+        const long long j = done + threadIdx.x;
+        P.in_mst[j] = (unsigned char)((P.mbits[j >> 5] >> (j & 31)) & 1u);
     }
 }
 

@@ -529,3 +529,23 @@ def test_populate_dynamic_tail_full_regions(eclmst, both, seed):
     assert stats["filtered"] == 1 and stats["phase2_round"] >= 0
     # phase 2 kept every canonical entry but the self-loops
     assert stats["live"][stats["phase2_round"]] == int((lo != hi).sum()) * (1 + both)
+
+
+@pytest.mark.parametrize("offset", [0, 4, 8, 12])
+def test_in_mst_alignment_and_poison(eclmst, offset):
+    """in_mst is written from the MSF bit marks at the end (k_expand): every
+    byte, 16 at a time where the output is 16-byte aligned and 4 at a time
+    otherwise (the C ABI asks for 4-byte alignment), plus a ragged tail
+    (M not a multiple of 16).  The output starts poisoned."""
+    g = G.random_small(3000, 40_001, seed=77, weights="ties", multi=True, self_loops=True)
+    omask, ototal, _ = oracle.kruskal_graph(g)
+    dev = torch.device("cuda:0")
+    gd = g.to(dev)
+    M = int(gd.nlist.numel())
+    assert M % 16 != 0
+    buf = torch.full((M + 64,), 0xAB, dtype=torch.uint8, device=dev)
+    out = buf[offset: offset + M]
+    mask, total, ws = eclmst.ecl_mst_device(gd.n, gd.nindex, gd.nlist, gd.eweight, in_mst_out=out)
+    assert int(total.item()) == ototal
+    assert np.array_equal(out.cpu().numpy(), omask)
+    assert (buf[:offset] == 0xAB).all() and (buf[offset + M:] == 0xAB).all()   # nothing outside
