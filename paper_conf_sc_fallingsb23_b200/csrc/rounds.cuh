@@ -9,6 +9,10 @@
 
 namespace eclmst {
 
+#ifndef ECL_WARP_CLAIM
+#define ECL_WARP_CLAIM 1   // k_rounds' warps take their CTA's chunks by a shared ticket (next_chunk)
+#endif
+
 // ---------------------------------------------------------------------------
 // k_flatten: set(v) for every vertex before the phase-2 populate, so
 // that populate reads each endpoint's set with one load.
@@ -286,13 +290,27 @@ __device__ __forceinline__ RegionSrcT<SOA> region_src(const Params& P, int b, in
 // level right before this pass, so the tuples still hold ids of the level
 // below, now closed: find() ends at the root's label, its id in the new level
 // (where nothing has hooked yet).  The tuples leave with the new level's ids.
+// Chunk order within the CTA (ECL_WARP_CLAIM): with a shared ticket counter
+// (s_tk, zero at the start of the pass) each warp takes the CTA's next chunk
+// when it is free, so the CTA's warps finish together instead of waiting at
+// the barrier for the one that drew the slow chunks; without it, warp w takes
+// chunks w, w + kWarps, ...  first_chunk/next_chunk return the next index or
+// a value >= nloc.
+__device__ __forceinline__ int next_chunk(int* s_tk, int k) {
+    if (!s_tk) return k + kWarps;
+    int t = 0;
+    if ((threadIdx.x & 31) == 0) t = atomicAdd(s_tk, 1);
+    return __shfl_sync(kFull, t, 0);
+}
+__device__ __forceinline__ int first_chunk(int* s_tk) { return s_tk ? next_chunk(s_tk, 0) : (int)(threadIdx.x >> 5); }
+
 template <bool SPLIT = false, bool MAP = false, class SRC>
 __device__ __forceinline__ void passA(const Params& P, const DS& D, const SRC& S, int4* __restrict__ out,
                                       int* s_out, bool guard, int T = INT_MAX, int4* out_end = nullptr,
-                                      int* s_def = nullptr) {
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+                                      int* s_def = nullptr, int* s_tk = nullptr) {
+    const int lane = threadIdx.x & 31;
     const bool halving = P.halving != 0;
-    for (int k = warp; k < S.nloc; k += kWarps) {
+    for (int k = first_chunk(s_tk); k < S.nloc; k = next_chunk(s_tk, k)) {
         int count;
         const int4* __restrict__ in = S.get(P, k, count);
         int4 t[kItems];
@@ -388,9 +406,10 @@ __device__ __forceinline__ void passA_vc(const Params& P, const DS& D, unsigned 
 // level's best-edge slots, so the winners leave them as they are (k_rounds
 // refills them should the relabel not happen after all).
 template <bool NORESET = false, class SRC>
-__device__ __forceinline__ void passB(const Params& P, const DS& D, const SRC& S, long long* acc) {
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    for (int kk = warp; kk < S.nloc; kk += kWarps) {
+__device__ __forceinline__ void passB(const Params& P, const DS& D, const SRC& S, long long* acc,
+                                      int* s_tk = nullptr) {
+    const int lane = threadIdx.x & 31;
+    for (int kk = first_chunk(s_tk); kk < S.nloc; kk = next_chunk(s_tk, kk)) {
         // (ECL_B_REVERSE: walk the chunks back to front, so pass B starts on the
         // tuples the last pass wrote most recently, still in L2, and the next
         // pass A, walking front to back, starts on the ones pass B read last)
@@ -730,7 +749,19 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
     __shared__ long long s_lv[4];
     __shared__ int s_lev;
     const DS D = ds_of(P);
+    // per-pass chunk tickets of this CTA's warps (next_chunk): pass i counts
+    // in s_tk[i & 1] and clears the other one, last used a barrier ago
+    __shared__ int s_tk[2];
+    int tkp = 0;
+    auto tk = [&]() -> int* {
+        if (!ECL_WARP_CLAIM) return nullptr;
+        int* c = &s_tk[tkp & 1];
+        if (tid == 0) s_tk[(tkp + 1) & 1] = 0;
+        ++tkp;
+        return c;
+    };
     if (tid == 0) {
+        s_tk[0] = 0;
         s_lev = __ldcg(&P.in->nlev);
         s_lv[0] = __ldcg(&P.in->lv_base);
         s_lv[1] = __ldcg(&P.in->lv_size);
@@ -753,8 +784,9 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
         // (both_directions: an edge's two copies must see the same slots, so
         // no copy resets them in pass B; the paper's separate reset kernel,
         // L34-37, follows instead)
-        if (noreset || P.both) passB<true>(P, D, S, acc);
-        else passB(P, D, S, acc);
+        int* const tkB = tk();
+        if (noreset || P.both) passB<true>(P, D, S, acc, tkB);
+        else passB(P, D, S, acc, tkB);
         const long long d = acc[1] - w0;
         if (lane == 0 && d) atomicAdd(reinterpret_cast<unsigned long long*>(&st->winners[g]), (unsigned long long)d);
         if (tid == 0) s_out = s_def = 0;
@@ -835,15 +867,17 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
             }
         }
         unsigned long long* const vcnt = &P.in->vc_cnt[g % 3];
+        int* const tkA = tk();
+        (void)tkA;
         if constexpr (vc) {
             if (b0 && tid == 0) P.in->vc_cnt[(g + 1) % 3] = 0;   // next round's list counter (read 2 rounds ago)
             passA_vc<PH, SOA>(P, D, vcnt, guard);
         } else if constexpr (topo) {
-            passA(P, D, R, wl[1], &s_out, guard);
+            passA(P, D, R, wl[1], &s_out, guard, INT_MAX, nullptr, nullptr, tkA);
         } else if (T != INT_MAX)
-            passA<true>(P, D, S, wl[cur ^ 1], &s_out, guard, T, tadd<SOA>(wl[cur ^ 1], P.cap), &s_def);
-        else if (mapped) passA<false, true>(P, D, S, wl[cur ^ 1], &s_out, guard);
-        else passA(P, D, S, wl[cur ^ 1], &s_out, guard);
+            passA<true>(P, D, S, wl[cur ^ 1], &s_out, guard, T, tadd<SOA>(wl[cur ^ 1], P.cap), &s_def, tkA);
+        else if (mapped) passA<false, true>(P, D, S, wl[cur ^ 1], &s_out, guard, INT_MAX, nullptr, nullptr, tkA);
+        else passA(P, D, S, wl[cur ^ 1], &s_out, guard, INT_MAX, nullptr, nullptr, tkA);
         cur = topo ? 1 : cur ^ 1;
         __syncthreads();
         C = compact_src<SOA>(wl[cur], s_out);
@@ -893,7 +927,7 @@ __global__ void __launch_bounds__(kBlock, ECL_R_MINB) k_rounds(Params P) {
             grid.sync();
         }
 #endif
-        passA(P, D, H, wl[ob], &s_out, true);
+        passA(P, D, H, wl[ob], &s_out, true, INT_MAX, nullptr, nullptr, tk());
         cur = ob;
         __syncthreads();
         C = compact_src<SOA>(wl[cur], s_out);
